@@ -1,0 +1,175 @@
+/*
+ * dtc.h -- C ABI of libdtc.so: the DTC-SpMM hot path on B200 (sm_100a).
+ *
+ * Operation: general unstructured SpMM  C(MxN) = A(MxK) * B(KxN)  with A sparse
+ * (§2.2), B and C dense row-major (§4.4.1), computed
+ * on tensor cores over the memory-efficient tensor-core format ME-TCF
+ * (§4.2) built from CSR on the GPU (§6).
+ * A fixed A is converted once and reused across many SpMM calls.
+ *
+ * Conventions (all entry points):
+ *  - Every function returns a dtc_status_t (0 = DTC_OK, negative = error).  No
+ *    exception or abort crosses the ABI; dtc_last_error() returns a thread-local
+ *    message with detail.
+ *  - Pointers are DEVICE pointers unless the name/comment says host.  Streams
+ *    are passed as `void*` holding a cudaStream_t (NULL = legacy default stream).
+ *  - The caller owns CSR, B and C.  The library owns everything reachable from a
+ *    handle (format arrays, schedule, workspaces) until *_destroy.
+ *  - There is no CPU fallback: without a CUDA device every compute call returns
+ *    DTC_ERR_CUDA.
+ */
+#ifndef DTC_H_
+#define DTC_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    DTC_OK = 0,
+    DTC_ERR_INVALID = -1,     /* bad argument / malformed rowptr              */
+    DTC_ERR_UNSORTED = -2,    /* CSR columns not ascending within a row       */
+    DTC_ERR_DUPLICATE = -3,   /* repeated column within a row                 */
+    DTC_ERR_RANGE = -4,       /* column index outside [0, K)                  */
+    DTC_ERR_OOM = -5,         /* device allocation failed                     */
+    DTC_ERR_CUDA = -6,        /* CUDA runtime error (incl. no device)         */
+    DTC_ERR_NCCL = -7,        /* NCCL error                                   */
+    DTC_ERR_UNSUPPORTED = -8  /* valid request this build does not handle     */
+} dtc_status_t;
+
+/* Value / operand precision.
+ * DTC_TF32: A values and B are fp32 in memory; the tensor cores multiply them
+ *           rounded to TF32 (cvt.rna) with fp32 accumulation.
+ * DTC_FP16: A values and B are fp16 in memory; fp32 accumulation; C is fp32.   */
+typedef enum { DTC_TF32 = 0, DTC_FP16 = 1 } dtc_dtype_t;
+
+/* Canonical CSR input (device pointers): rowptr int32[M+1] with rowptr[0]=0,
+ * rowptr[M]=nnz, non-decreasing; colidx int32[nnz] strictly increasing within a
+ * row and in [0,K); vals[nnz] of `dtype` (fp32 or fp16).  nnz < 2^31.
+ * Explicit zeros are structural non-zeros and are kept. */
+typedef struct {
+    int64_t M, K, nnz;
+    const int32_t* rowptr;
+    const int32_t* colidx;
+    const void* vals;
+    int32_t dtype;            /* dtc_dtype_t */
+} dtc_csr_t;
+
+typedef struct dtc_format* dtc_handle_t;   /* opaque, library-owned */
+
+/* Borrowed device views of the ME-TCF arrays, valid until
+ * dtc_format_destroy:
+ *   row_window_offset int32[num_windows+1]  start TC block of each 16-row window
+ *   tc_offset         int32[T+1]            start of each TC block in tc_local_id
+ *   tc_local_id       uint8[nnz]            row_in_window*8 + col_in_block (<128)
+ *   sparse_a_to_b     int32[8T]             original column of each block column, -1 pad
+ *   tc_values         dtype[nnz]            values aligned with tc_local_id
+ *   units             int32[8*num_units]    F4 work-unit table (see dtc_schedule_export) */
+typedef struct {
+    int64_t M, K, nnz, num_windows, num_tc_blocks, num_units, num_split_windows;
+    int32_t dtype;
+    int32_t unit_blocks;
+    const int32_t* row_window_offset;
+    const int32_t* tc_offset;
+    const uint8_t* tc_local_id;
+    const int32_t* sparse_a_to_b;
+    const void* tc_values;
+    const int32_t* units;
+} dtc_format_view_t;
+
+/* Build options (zero-initialised = defaults).
+ *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T and the SM count
+ *   dedup_path   F1 per-window dedup: 0 auto, 1 force smem sort, 2 force chunked bitmap
+ *                (both produce bit-identical formats; exposed for tests) */
+typedef struct {
+    int32_t unit_blocks;
+    int32_t dedup_path;
+} dtc_build_opts_t;
+
+/* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on
+ * the GPU.  Stream-ordered; blocks on `stream`
+ * twice (to read NumTCBlock + the validation flag, and the unit count) in
+ * order to size allocations.  On error *out is NULL and nothing leaks.
+ * Errors: INVALID (null/negative sizes, malformed rowptr), UNSORTED, DUPLICATE,
+ * RANGE, OOM, CUDA. */
+int dtc_format_build(const dtc_csr_t* csr, void* stream, dtc_handle_t* out);
+int dtc_format_build_ex(const dtc_csr_t* csr, const dtc_build_opts_t* opts, void* stream,
+                        dtc_handle_t* out);
+
+/* Fill *view with borrowed device pointers and sizes.  INVALID if h or view is NULL. */
+int dtc_format_query(dtc_handle_t h, dtc_format_view_t* view);
+
+/* Copy the ME-TCF arrays to HOST buffers (any pointer may be NULL to skip it):
+ * rwo int32[W+1], tco int32[T+1], lid uint8[nnz], atob int32[8T],
+ * vals dtype[nnz], units int32[8*num_units].  Synchronous. */
+int dtc_format_export(dtc_handle_t h, int32_t* rwo, int32_t* tco, uint8_t* lid, int32_t* atob,
+                      void* vals, int32_t* units);
+
+/* S1-S5: C := A*B (kernel design PAPER.md:260-333, re-designed for
+ * sm_100a).  B: device, K x N row-major with row stride ldb >= N, dtype of the
+ * handle.  C: device fp32, M x N row-major with ldc >= N; every element of the
+ * M x N region is overwritten (empty rows -> 0).  N >= 1.  Asynchronous on
+ * `stream`; deterministic (bit-identical run to run).  16-byte aligned B/C with
+ * ldb, ldc, N multiples of 16/sizeof(elt) take the vector path, anything else the
+ * scalar path.  Concurrent dtc_spmm calls on ONE handle must be stream-ordered
+ * (they share the split-window workspace).  Errors: INVALID, CUDA, OOM. */
+int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc,
+             void* stream);
+
+/* End-to-end variant with HOST buffers: copies B (host, K x N, ldb) to a
+ * library-owned device buffer, runs dtc_spmm, copies C back to host (M x N,
+ * ldc) and synchronises `stream`.  Pinned host memory gives full PCIe/C2C rate. */
+int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
+                  int64_t ldc, void* stream);
+
+/* Number of kernels dtc_spmm launches per call (for launch accounting). */
+int dtc_spmm_launches_per_call(void);
+
+void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory */
+
+/* ------------------------------------------------------------ distributed
+ * One process per GPU (north_star).  Row windows are partitioned across ranks
+ * into contiguous ranges balanced by TC-block count; every rank needs all of B,
+ * which the root broadcasts with NCCL; C can be all-gathered. */
+typedef struct dtc_dist* dtc_dist_t;
+
+/* HOST, pure: split windows [0,W) into `world` contiguous ranges at the smallest
+ * w with rwo[w] >= r*T/world (r = 1..world-1).  w_begin int64[world+1].
+ * Callable without a GPU.  INVALID on bad sizes. */
+int dtc_partition_windows(const int32_t* rwo_host, int64_t num_windows, int32_t world,
+                          int64_t* w_begin);
+
+/* Write a fresh 128-byte NCCL unique id to out128 (host). */
+int dtc_nccl_unique_id(void* out128);
+
+/* Collective over `world` ranks: condense the FULL csr (device pointers on this
+ * rank's GPU) to find the window partition, then build this rank's local ME-TCF
+ * from its CSR row slice.  nccl_id (host, 128 B, identical on all ranks) may be
+ * NULL for a communicator-less local shard (single-GPU shard tests). */
+int dtc_dist_create(const dtc_csr_t* csr_full, int32_t rank, int32_t world, const void* nccl_id,
+                    void* stream, dtc_dist_t* out);
+
+/* This rank's C rows [row_begin, row_end) and its local format handle (borrowed). */
+int dtc_dist_query(dtc_dist_t d, int64_t* row_begin, int64_t* row_end, dtc_handle_t* local);
+
+/* B: device K x N (ldb = N), valid on `root` (broadcast in place to the others).
+ * C: device fp32; if gather_c, M x N (ldc = N) and every rank receives all rows;
+ * else this rank's (row_end-row_begin) x N rows.  Needs a communicator unless
+ * world == 1.  Stream-ordered.  Errors: INVALID, NCCL, CUDA. */
+int dtc_spmm_dist(dtc_dist_t d, void* B, int32_t root, int64_t N, float* C, int32_t gather_c,
+                  void* stream);
+
+void dtc_dist_destroy(dtc_dist_t d);
+
+/* ------------------------------------------------------------ diagnostics */
+const char* dtc_status_string(int status);
+const char* dtc_last_error(void);
+/* Library build string (arch, version). */
+const char* dtc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DTC_H_ */

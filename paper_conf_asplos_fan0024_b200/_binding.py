@@ -1,0 +1,307 @@
+"""ctypes marshalling for include/dtc.h.  No computation happens here."""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libdtc.so")
+_HEADER = os.path.join(os.path.dirname(_HERE), "include", "dtc.h")
+
+DTC_OK = 0
+DTC_ERR_INVALID = -1
+DTC_ERR_UNSORTED = -2
+DTC_ERR_DUPLICATE = -3
+DTC_ERR_RANGE = -4
+DTC_ERR_OOM = -5
+DTC_ERR_CUDA = -6
+DTC_ERR_NCCL = -7
+DTC_ERR_UNSUPPORTED = -8
+DTC_TF32 = 0
+DTC_FP16 = 1
+
+_i64, _i32, _vp = ctypes.c_int64, ctypes.c_int32, ctypes.c_void_p
+
+
+class _Csr(ctypes.Structure):
+    _fields_ = [("M", _i64), ("K", _i64), ("nnz", _i64), ("rowptr", _vp), ("colidx", _vp),
+                ("vals", _vp), ("dtype", _i32)]
+
+
+class _View(ctypes.Structure):
+    _fields_ = [("M", _i64), ("K", _i64), ("nnz", _i64), ("num_windows", _i64), ("num_tc_blocks", _i64),
+                ("num_units", _i64), ("num_split_windows", _i64), ("dtype", _i32), ("unit_blocks", _i32),
+                ("row_window_offset", _vp), ("tc_offset", _vp), ("tc_local_id", _vp),
+                ("sparse_a_to_b", _vp), ("tc_values", _vp), ("units", _vp)]
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32)]
+
+
+class DtcError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        self.status = status
+        super().__init__(f"{where}: {_status_name(status)} ({status}): {detail}")
+
+
+_lock = threading.Lock()
+_lib = None
+
+
+def library_path() -> str:
+    return _SO
+
+
+def lib():
+    """Load libdtc.so; raise loudly if it has not been built (no fallback)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(_SO):
+                raise ImportError(f"{_SO} is missing: build it with `python -c 'import __graft_entry__ as g; "
+                                  f"g.build()'` (there is no CPU fallback)")
+            L = ctypes.CDLL(_SO)
+            P = ctypes.POINTER
+            L.dtc_format_build.argtypes = [P(_Csr), _vp, P(_vp)]
+            L.dtc_format_build_ex.argtypes = [P(_Csr), P(_Opts), _vp, P(_vp)]
+            L.dtc_format_query.argtypes = [_vp, P(_View)]
+            L.dtc_format_export.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp]
+            L.dtc_spmm.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
+            L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
+            L.dtc_spmm_launches_per_call.argtypes = []
+            L.dtc_format_destroy.argtypes = [_vp]
+            L.dtc_format_destroy.restype = None
+            L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
+            L.dtc_nccl_unique_id.argtypes = [_vp]
+            L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
+            L.dtc_dist_query.argtypes = [_vp, P(_i64), P(_i64), P(_vp)]
+            L.dtc_spmm_dist.argtypes = [_vp, _vp, _i32, _i64, _vp, _i32, _vp]
+            L.dtc_dist_destroy.argtypes = [_vp]
+            L.dtc_dist_destroy.restype = None
+            L.dtc_status_string.argtypes = [ctypes.c_int]
+            L.dtc_status_string.restype = ctypes.c_char_p
+            L.dtc_last_error.argtypes = []
+            L.dtc_last_error.restype = ctypes.c_char_p
+            L.dtc_version.argtypes = []
+            L.dtc_version.restype = ctypes.c_char_p
+            _lib = L
+    return _lib
+
+
+def _status_name(st: int) -> str:
+    try:
+        return lib().dtc_status_string(st).decode()
+    except Exception:
+        return str(st)
+
+
+def _check(st: int, where: str):
+    if st != DTC_OK:
+        raise DtcError(st, where, lib().dtc_last_error().decode())
+
+
+def exported_symbols() -> list[str]:
+    """Function names declared in include/dtc.h."""
+    txt = open(_HEADER).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(dtc_[a-z0-9_]+)\s*\(", txt)))
+
+
+def version() -> str:
+    return lib().dtc_version().decode()
+
+
+def launches_per_call() -> int:
+    return int(lib().dtc_spmm_launches_per_call())
+
+
+def _dtype_code(dtype) -> int:
+    if dtype in ("tf32", "fp32", DTC_TF32):
+        return DTC_TF32
+    if dtype in ("fp16", "f16", DTC_FP16):
+        return DTC_FP16
+    raise ValueError(f"dtype {dtype!r}")
+
+
+def _stream_ptr(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _dptr(t) -> int:
+    return 0 if t is None else int(t.data_ptr())
+
+
+def _make_csr(rowptr, colidx, vals, M, K, dtype) -> _Csr:
+    import torch
+    code = _dtype_code(dtype)
+    for name, t, dt in (("rowptr", rowptr, torch.int32), ("colidx", colidx, torch.int32)):
+        if t.dtype != dt or not t.is_cuda or not t.is_contiguous():
+            raise TypeError(f"{name} must be a contiguous CUDA int32 tensor")
+    want = torch.float16 if code == DTC_FP16 else torch.float32
+    if vals.dtype != want or not vals.is_cuda or not vals.is_contiguous():
+        raise TypeError(f"vals must be a contiguous CUDA {want} tensor")
+    return _Csr(int(M), int(K), int(colidx.numel()), _dptr(rowptr), _dptr(colidx), _dptr(vals), code)
+
+
+class Format:
+    """An ME-TCF handle (library-owned device memory)."""
+
+    def __init__(self, handle: int, keep=()):
+        self._h = ctypes.c_void_p(handle)
+        self._keep = keep
+        v = self.query()
+        self.M, self.K, self.nnz = v.M, v.K, v.nnz
+        self.num_windows, self.num_tc_blocks = v.num_windows, v.num_tc_blocks
+        self.num_units, self.num_split_windows = v.num_units, v.num_split_windows
+        self.unit_blocks = v.unit_blocks
+        self.dtype = "fp16" if v.dtype == DTC_FP16 else "tf32"
+
+    @classmethod
+    def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
+              unit_blocks: int = 0, dedup_path: int = 0) -> "Format":
+        csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
+        h = ctypes.c_void_p()
+        opts = _Opts(int(unit_blocks), int(dedup_path))
+        _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
+                                         ctypes.byref(h)), "dtc_format_build")
+        return cls(h.value)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def query(self) -> _View:
+        v = _View()
+        _check(lib().dtc_format_query(self._h, ctypes.byref(v)), "dtc_format_query")
+        return v
+
+    def export(self) -> dict:
+        """Copy the ME-TCF arrays to host numpy arrays (bit-exact checks)."""
+        W, T, nnz, nu = self.num_windows, self.num_tc_blocks, self.nnz, self.num_units
+        out = {
+            "row_window_offset": np.zeros(W + 1, np.int32),
+            "tc_offset": np.zeros(T + 1, np.int32),
+            "tc_local_id": np.zeros(max(nnz, 1), np.uint8),
+            "sparse_a_to_b": np.zeros(max(8 * T, 1), np.int32),
+            "tc_values": np.zeros(max(nnz, 1), np.float16 if self.dtype == "fp16" else np.float32),
+            "units": np.zeros((max(nu, 1), 8), np.int32),
+        }
+        p = {k: v.ctypes.data_as(_vp) for k, v in out.items()}
+        _check(lib().dtc_format_export(self._h, p["row_window_offset"], p["tc_offset"], p["tc_local_id"],
+                                       p["sparse_a_to_b"], p["tc_values"], p["units"]), "dtc_format_export")
+        out["tc_local_id"] = out["tc_local_id"][:nnz]
+        out["tc_values"] = out["tc_values"][:nnz]
+        out["sparse_a_to_b"] = out["sparse_a_to_b"][: 8 * T]
+        out["units"] = out["units"][:nu]
+        out["num_windows"] = W
+        out["num_tc_blocks"] = T
+        return out
+
+    def spmm(self, B, C=None, stream=None):
+        """C := A @ B on the GPU (B: CUDA tensor K x N of the handle dtype, row stride ldb)."""
+        import torch
+        if B.dim() != 2 or not B.is_cuda or B.stride(1) != 1:
+            raise TypeError("B must be a 2-D CUDA tensor with unit column stride")
+        want = torch.float16 if self.dtype == "fp16" else torch.float32
+        if B.dtype != want:
+            raise TypeError(f"B must be {want}")
+        N = B.shape[1]
+        if C is None:
+            C = torch.empty((self.M, N), dtype=torch.float32, device=B.device)
+        if C.dtype != torch.float32 or C.stride(1) != 1 or C.shape[0] != self.M or C.shape[1] != N:
+            raise TypeError("C must be a float32 (M x N) CUDA tensor with unit column stride")
+        _check(lib().dtc_spmm(self._h, _dptr(B), N, B.stride(0), _dptr(C), C.stride(0), _stream_ptr(stream)),
+               "dtc_spmm")
+        return C
+
+    def spmm_raw(self, B_ptr: int, N: int, ldb: int, C_ptr: int, ldc: int, stream=None):
+        _check(lib().dtc_spmm(self._h, B_ptr, N, ldb, C_ptr, ldc, _stream_ptr(stream)), "dtc_spmm")
+
+    def spmm_host(self, B_host, C_host=None, stream=None):
+        """End-to-end C = A @ B with HOST buffers (numpy or pinned torch CPU tensors)."""
+        bp, N, ldb = _host_ptr(B_host)
+        if C_host is None:
+            C_host = np.empty((self.M, N), dtype=np.float32)
+        cp, _, ldc = _host_ptr(C_host)
+        _check(lib().dtc_spmm_host(self._h, bp, N, ldb, cp, ldc, _stream_ptr(stream)), "dtc_spmm_host")
+        return C_host
+
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib().dtc_format_destroy(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _host_ptr(a):
+    if isinstance(a, np.ndarray):
+        assert a.ndim == 2 and a.strides[1] == a.itemsize
+        return a.ctypes.data, a.shape[1], a.strides[0] // a.itemsize
+    # torch CPU tensor
+    assert a.dim() == 2 and a.stride(1) == 1 and not a.is_cuda
+    return a.data_ptr(), a.shape[1], a.stride(0)
+
+
+def partition_windows(rwo, world: int) -> np.ndarray:
+    """Host-side window partition by TC-block prefix (dtc_partition_windows)."""
+    rwo = np.ascontiguousarray(rwo, dtype=np.int32)
+    out = np.zeros(world + 1, dtype=np.int64)
+    _check(lib().dtc_partition_windows(rwo.ctypes.data_as(_vp), len(rwo) - 1, world, out.ctypes.data_as(_vp)),
+           "dtc_partition_windows")
+    return out
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().dtc_nccl_unique_id(buf), "dtc_nccl_unique_id")
+    return buf.raw
+
+
+class Dist:
+    """One rank's share of a row-window-partitioned SpMM (dtc_dist_*)."""
+
+    def __init__(self, rowptr, colidx, vals, M, K, dtype, rank: int, world: int, nccl_id: bytes | None,
+                 stream=None):
+        csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
+        h = ctypes.c_void_p()
+        idbuf = ctypes.create_string_buffer(nccl_id, 128) if nccl_id is not None else None
+        _check(lib().dtc_dist_create(ctypes.byref(csr), rank, world, idbuf, _stream_ptr(stream), ctypes.byref(h)),
+               "dtc_dist_create")
+        self._h = h
+        self.M, self.K, self.rank, self.world = M, K, rank, world
+        self.dtype = "fp16" if _dtype_code(dtype) == DTC_FP16 else "tf32"
+        rb, re_, loc = _i64(), _i64(), _vp()
+        _check(lib().dtc_dist_query(self._h, ctypes.byref(rb), ctypes.byref(re_), ctypes.byref(loc)),
+               "dtc_dist_query")
+        self.row_begin, self.row_end = rb.value, re_.value
+
+    def spmm(self, B, C, root: int = 0, gather_c: bool = True, stream=None):
+        N = B.shape[1]
+        assert B.is_contiguous() and C.is_contiguous()
+        _check(lib().dtc_spmm_dist(self._h, _dptr(B), root, N, _dptr(C), int(gather_c), _stream_ptr(stream)),
+               "dtc_spmm_dist")
+        return C
+
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib().dtc_dist_destroy(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,168 @@
+// dtc_dist.cu -- multi-GPU row-window data parallelism (north_star; the paper is
+// single-GPU, its parallelism is row windows across SMs).
+//
+// One process per GPU.  Windows are split into contiguous ranges balanced by
+// TC-block count (prefix of RowWindowOffset); each rank condenses only its CSR
+// row slice.  The single exchange is B: every rank needs all of it because the
+// columns of A are arbitrary, so the root broadcasts it with NCCL over
+// NVLink/NVSwitch.  C can be all-gathered (each owner broadcasts its rows,
+// grouped), otherwise each rank keeps its own rows.
+#include <nccl.h>
+
+#include <new>
+#include <vector>
+
+#include "dtc_internal.h"
+
+struct dtc_dist {
+    int rank = 0, world = 1;
+    int64_t M = 0, K = 0;
+    int32_t dtype = 0;
+    std::vector<int64_t> row_begin;  // [world+1]
+    dtc_format* local = nullptr;
+    int32_t* local_rowptr = nullptr;
+    ncclComm_t comm = nullptr;
+};
+
+namespace dtc {
+
+static int nccl_fail(ncclResult_t r, const char* what) {
+    set_error("%s failed: %s", what, ncclGetErrorString(r));
+    return DTC_ERR_NCCL;
+}
+#define DTC_NCCL(call)                                              \
+    do {                                                            \
+        ncclResult_t _r = (call);                                   \
+        if (_r != ncclSuccess) return ::dtc::nccl_fail(_r, #call);  \
+    } while (0)
+
+__global__ void k_rebase(const int32_t* __restrict__ in, int32_t* __restrict__ out, int64_t n, int32_t base) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = in[i] - base;
+}
+
+}  // namespace dtc
+
+using namespace dtc;
+
+extern "C" int dtc_partition_windows(const int32_t* rwo, int64_t W, int32_t world, int64_t* w_begin) {
+    if (!rwo || !w_begin || W < 0 || world < 1) { set_error("bad partition arguments"); return DTC_ERR_INVALID; }
+    const int64_t T = rwo[W];
+    w_begin[0] = 0;
+    int64_t w = 0;
+    for (int r = 1; r < world; ++r) {
+        // smallest w with rwo[w] >= r*T/world (ceil), never before the previous cut
+        const int64_t target = (T * r + world - 1) / world;
+        while (w < W && rwo[w] < target) ++w;
+        w_begin[r] = w;
+    }
+    w_begin[world] = W;
+    return DTC_OK;
+}
+
+extern "C" int dtc_nccl_unique_id(void* out128) {
+    if (!out128) { set_error("null output"); return DTC_ERR_INVALID; }
+    ncclUniqueId id;
+    DTC_NCCL(ncclGetUniqueId(&id));
+    static_assert(sizeof(ncclUniqueId) == 128, "NCCL unique id is 128 bytes");
+    memcpy(out128, &id, sizeof(id));
+    return DTC_OK;
+}
+
+extern "C" int dtc_dist_create(const dtc_csr_t* csr, int32_t rank, int32_t world, const void* nccl_id, void* stream,
+                               dtc_dist_t* out) {
+    if (!out) { set_error("out is NULL"); return DTC_ERR_INVALID; }
+    *out = nullptr;
+    if (!csr || world < 1 || rank < 0 || rank >= world) { set_error("bad rank/world"); return DTC_ERR_INVALID; }
+    cudaStream_t s = (cudaStream_t)stream;
+    // 1. window partition from the full matrix's RowWindowOffset
+    dtc_format* full = nullptr;
+    int rc = format_build(csr, nullptr, s, &full);
+    if (rc) return rc;
+    std::vector<int32_t> rwo(full->W + 1);
+    cudaError_t e = cudaMemcpy(rwo.data(), full->rwo, (full->W + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost);
+    dtc_format_destroy(full);
+    if (e != cudaSuccess) return cuda_fail(e, "rwo readback", __FILE__, __LINE__);
+    std::vector<int64_t> wb(world + 1);
+    dtc_partition_windows(rwo.data(), (int64_t)rwo.size() - 1, world, wb.data());
+    dtc_dist* d = new (std::nothrow) dtc_dist();
+    if (!d) { set_error("host OOM"); return DTC_ERR_OOM; }
+    d->rank = rank; d->world = world; d->M = csr->M; d->K = csr->K; d->dtype = csr->dtype;
+    d->row_begin.resize(world + 1);
+    for (int r = 0; r <= world; ++r) d->row_begin[r] = std::min<int64_t>(wb[r] * kWindow, csr->M);
+    // 2. local CSR slice (rows [r0, r1)), rowptr rebased to 0
+    const int64_t r0 = d->row_begin[rank], r1 = d->row_begin[rank + 1];
+    int32_t base = 0, endp = 0;
+    if (csr->M > 0) {
+        e = cudaMemcpy(&base, csr->rowptr + r0, sizeof(int32_t), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(&endp, csr->rowptr + r1, sizeof(int32_t), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) { delete d; return cuda_fail(e, "rowptr readback", __FILE__, __LINE__); }
+    }
+    rc = dalloc(&d->local_rowptr, r1 - r0 + 1, s);
+    if (rc) { delete d; return rc; }
+    k_rebase<<<64, 256, 0, s>>>(csr->rowptr + r0, d->local_rowptr, r1 - r0 + 1, base);
+    dtc_csr_t lc;
+    lc.M = r1 - r0; lc.K = csr->K; lc.nnz = endp - base;
+    lc.rowptr = d->local_rowptr;
+    lc.colidx = csr->colidx + base;
+    lc.vals = (const char*)csr->vals + (int64_t)base * elt_size(csr->dtype);
+    lc.dtype = csr->dtype;
+    rc = format_build(&lc, nullptr, s, &d->local);
+    if (rc) { dfree(d->local_rowptr, s); cudaStreamSynchronize(s); delete d; return rc; }
+    // 3. communicator
+    if (nccl_id && world > 1) {
+        ncclUniqueId id;
+        memcpy(&id, nccl_id, sizeof(id));
+        ncclResult_t nr = ncclCommInitRank(&d->comm, world, id, rank);
+        if (nr != ncclSuccess) {
+            dtc_format_destroy(d->local);
+            dfree(d->local_rowptr, s);
+            cudaStreamSynchronize(s);
+            delete d;
+            return nccl_fail(nr, "ncclCommInitRank");
+        }
+    }
+    *out = d;
+    return DTC_OK;
+}
+
+extern "C" int dtc_dist_query(dtc_dist_t d, int64_t* row_begin, int64_t* row_end, dtc_handle_t* local) {
+    if (!d) { set_error("null dist"); return DTC_ERR_INVALID; }
+    if (row_begin) *row_begin = d->row_begin[d->rank];
+    if (row_end) *row_end = d->row_begin[d->rank + 1];
+    if (local) *local = d->local;
+    return DTC_OK;
+}
+
+extern "C" int dtc_spmm_dist(dtc_dist_t d, void* B, int32_t root, int64_t N, float* C, int32_t gather_c,
+                             void* stream) {
+    if (!d || !C || N < 1 || root < 0 || root >= d->world) { set_error("bad dist arguments"); return DTC_ERR_INVALID; }
+    if (d->world > 1 && !d->comm) { set_error("no communicator (created with nccl_id == NULL)"); return DTC_ERR_INVALID; }
+    cudaStream_t s = (cudaStream_t)stream;
+    const ncclDataType_t bt = d->dtype == DTC_FP16 ? ncclHalf : ncclFloat;
+    if (d->world > 1 && d->K > 0) DTC_NCCL(ncclBroadcast(B, B, (size_t)(d->K * N), bt, root, d->comm, s));
+    const int64_t r0 = d->row_begin[d->rank];
+    float* Cl = gather_c ? C + r0 * N : C;
+    int rc = spmm_launch(d->local, B, N, N, Cl, N, s);
+    if (rc) return rc;
+    if (gather_c && d->world > 1) {
+        DTC_NCCL(ncclGroupStart());
+        for (int r = 0; r < d->world; ++r) {
+            const int64_t a = d->row_begin[r], b = d->row_begin[r + 1];
+            if (b > a) {
+                float* p = C + a * N;
+                DTC_NCCL(ncclBroadcast(p, p, (size_t)((b - a) * N), ncclFloat, r, d->comm, s));
+            }
+        }
+        DTC_NCCL(ncclGroupEnd());
+    }
+    return DTC_OK;
+}
+
+extern "C" void dtc_dist_destroy(dtc_dist_t d) {
+    if (!d) return;
+    if (d->comm) ncclCommDestroy(d->comm);
+    dtc_format_destroy(d->local);
+    if (d->local_rowptr) { cudaFree(d->local_rowptr); d->local_rowptr = nullptr; }
+    delete d;
+}

@@ -1,0 +1,594 @@
+// dtc_format.cu -- F0-F4: CSR -> ME-TCF condensation and the work-unit schedule,
+// all on the GPU ("Modules ... accelerated by highly parallel CUDA
+// kernels", :457 "we develop GPU kernels to accelerate this process").
+//
+// ME-TCF (§4.2): RowWindowOffset[W+1], TCOffset[T+1],
+// TCLocalId[nnz] (uint8), SparseAtoB[8T]; plus TCValues[nnz] (C7).
+// Canonical form (C3-C6): a window's condensed columns are its unique
+// original columns in ascending order; local id = row_in_window*8 + col_in_block;
+// the nnz of a block are stored by ascending local id; the last block of a
+// window is padded with -1.
+//
+// Pipeline:
+//   F0  k_validate        warp per row: rowptr shape, column range/order/dupes
+//   F1  k_dedup_sort      CTA per window with <= 2048 nnz: smem bitonic sort + unique
+//       k_dedup_bitmap    CTA per larger window: chunked smem bitmap over its column span
+//                         -> u_w, the window's ascending unique list, rank of every nnz
+//   F2  scan ceil(u_w/8)  -> RowWindowOffset, T                  (host sync #1)
+//   F3  k_fill_atob, k_mask (128-bit occupancy per TC block), k_blkcnt + scan ->
+//       TCOffset, k_place (position = TCOffset + popcount of lower ids)
+//   F4  k_units_count + scans + k_units_fill/fix (host sync #2: unit count)
+#include <algorithm>
+#include <climits>
+#include <cstring>
+#include <new>
+
+#include "dtc_device.cuh"
+#include "dtc_internal.h"
+
+namespace dtc {
+
+constexpr int kSortMax = 2048;         // windows up to this many nnz take the smem sort path
+constexpr int kSortThreads = 256;
+constexpr int kBmThreads = 256;
+constexpr int kBmWords = 8192;          // 2^18 columns per bitmap chunk
+constexpr int kBmBits = kBmWords * 32;
+
+enum : int { F_INVALID = 1, F_UNSORTED = 2, F_DUPLICATE = 4, F_RANGE = 8 };
+
+__device__ __forceinline__ int64_t clamp64(int64_t v, int64_t lo, int64_t hi) {
+    return v < lo ? lo : (v > hi ? hi : v);
+}
+
+// Window w's nnz segment [s0, s1) (clamped so malformed input cannot fault).
+__device__ __forceinline__ void window_segment(const int32_t* rowptr, int64_t M, int64_t nnz, int64_t w,
+                                               int64_t* s0, int64_t* s1) {
+    int64_t r0 = w * kWindow, r1 = min(r0 + kWindow, M);
+    int64_t a = clamp64(rowptr[r0], 0, nnz), b = clamp64(rowptr[r1], 0, nnz);
+    *s0 = a;
+    *s1 = b < a ? a : b;
+}
+
+// ---------------------------------------------------------------- F0
+__global__ void k_validate(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowptr,
+                           const int32_t* __restrict__ colidx, int* __restrict__ flags) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    int f = 0;
+    for (int64_t r = warp; r < M; r += nwarps) {
+        int64_t lo = rowptr[r], hi = rowptr[r + 1];
+        if ((r == 0 && lo != 0) || (r == M - 1 && hi != nnz) || lo < 0 || hi > nnz || lo > hi) {
+            f |= F_INVALID;
+            continue;
+        }
+        for (int64_t p = lo + lane; p < hi; p += 32) {
+            int c = colidx[p];
+            if (c < 0 || c >= K) f |= F_RANGE;
+            if (p > lo) {
+                int prev = colidx[p - 1];
+                if (c == prev) f |= F_DUPLICATE;
+                else if (c < prev) f |= F_UNSORTED;
+            }
+        }
+    }
+    f = __reduce_or_sync(0xffffffffu, f);
+    if (lane == 0 && f) atomicOr(flags, f);
+}
+
+// ---------------------------------------------------------------- F1 (sort path)
+// Output per window: u[w] (unique count), nb[w] = ceil(u/8), uniq[s0 + k] (k < u)
+// ascending unique columns, rank[p] for p in the segment.
+__global__ void __launch_bounds__(kSortThreads)
+k_dedup_sort(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowptr,
+             const int32_t* __restrict__ colidx, int mode, int32_t* __restrict__ u_out,
+             int64_t* __restrict__ nb_out, int32_t* __restrict__ uniq, int32_t* __restrict__ rank) {
+    __shared__ int s_key[kSortMax];
+    __shared__ int s_u[kSortMax];
+    const int64_t w = blockIdx.x;
+    int64_t s0, s1;
+    window_segment(rowptr, M, nnz, w, &s0, &s1);
+    const int64_t n64 = s1 - s0;
+    const int n = n64 > INT_MAX ? INT_MAX : (int)n64;
+    if (n > kSortMax || mode == 2) return;  // bitmap path handles it
+    if (n == 0) {
+        if (threadIdx.x == 0) { u_out[w] = 0; nb_out[w] = 0; }
+        return;
+    }
+    int P = 32;
+    while (P < n) P <<= 1;
+    for (int i = threadIdx.x; i < P; i += kSortThreads) s_key[i] = i < n ? colidx[s0 + i] : INT_MAX;
+    __syncthreads();
+    for (int k = 2; k <= P; k <<= 1) {
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = threadIdx.x; i < P; i += kSortThreads) {
+                int ixj = i ^ j;
+                if (ixj > i) {
+                    int a = s_key[i], b = s_key[ixj];
+                    bool up = (i & k) == 0;
+                    if ((a > b) == up) { s_key[i] = b; s_key[ixj] = a; }
+                }
+            }
+            __syncthreads();
+        }
+    }
+    // unique compaction: each thread owns a contiguous run of ITEMS keys
+    constexpr int ITEMS = kSortMax / kSortThreads;
+    const int i0 = threadIdx.x * ITEMS;
+    int cnt = 0;
+#pragma unroll
+    for (int q = 0; q < ITEMS; ++q) {
+        int i = i0 + q;
+        if (i < n && (i == 0 || s_key[i] != s_key[i - 1])) ++cnt;
+    }
+    int total;
+    int pos = block_exscan<kSortThreads>(cnt, &total);
+#pragma unroll
+    for (int q = 0; q < ITEMS; ++q) {
+        int i = i0 + q;
+        if (i < n && (i == 0 || s_key[i] != s_key[i - 1])) {
+            s_u[pos] = s_key[i];
+            uniq[s0 + pos] = s_key[i];
+            ++pos;
+        }
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < n; i += kSortThreads) {
+        int c = colidx[s0 + i];
+        int lo = 0, hi = total;
+        while (lo < hi) {
+            int mid = (lo + hi) >> 1;
+            if (s_u[mid] < c) lo = mid + 1; else hi = mid;
+        }
+        rank[s0 + i] = lo;
+    }
+    if (threadIdx.x == 0) {
+        u_out[w] = total;
+        nb_out[w] = (total + kTcw - 1) / kTcw;
+    }
+}
+
+// ---------------------------------------------------------------- F1 (bitmap path)
+__global__ void __launch_bounds__(kBmThreads)
+k_dedup_bitmap(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowptr,
+               const int32_t* __restrict__ colidx, int mode, int32_t* __restrict__ u_out,
+               int64_t* __restrict__ nb_out, int32_t* __restrict__ uniq, int32_t* __restrict__ rank) {
+    extern __shared__ uint32_t smem_bm[];
+    uint32_t* bm = smem_bm;                 // [kBmWords]
+    int* pref = (int*)(smem_bm + kBmWords); // [kBmWords] exclusive popcount prefix
+    const int64_t w = blockIdx.x;
+    int64_t s0, s1;
+    window_segment(rowptr, M, nnz, w, &s0, &s1);
+    const int64_t n = s1 - s0;
+    if (mode != 2 && n <= kSortMax) return;  // sort path handled it
+    int lo = INT_MAX, hi = -1;
+    for (int64_t p = s0 + threadIdx.x; p < s1; p += kBmThreads) {
+        int c = colidx[p];
+        if (c >= 0 && c < K) { lo = min(lo, c); hi = max(hi, c); }
+    }
+    lo = block_min<kBmThreads>(lo);
+    hi = block_max<kBmThreads>(hi);
+    int64_t base_rank = 0;
+    constexpr int WPT = kBmWords / kBmThreads;  // words per thread in the scan
+    for (int64_t c0 = lo; c0 <= hi; c0 += kBmBits) {
+        for (int i = threadIdx.x; i < kBmWords; i += kBmThreads) bm[i] = 0u;
+        __syncthreads();
+        for (int64_t p = s0 + threadIdx.x; p < s1; p += kBmThreads) {
+            int64_t c = colidx[p];
+            if (c >= c0 && c < c0 + kBmBits && c < K) {
+                int off = (int)(c - c0);
+                atomicOr(&bm[off >> 5], 1u << (off & 31));
+            }
+        }
+        __syncthreads();
+        int my = 0;
+        const int wb = threadIdx.x * WPT;
+#pragma unroll 8
+        for (int q = 0; q < WPT; ++q) my += __popc(bm[wb + q]);
+        int chunk_total;
+        int run = block_exscan<kBmThreads>(my, &chunk_total);
+        for (int q = 0; q < WPT; ++q) {
+            uint32_t bits = bm[wb + q];
+            pref[wb + q] = run;
+            int k = 0;
+            while (bits) {
+                int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                uniq[s0 + base_rank + run + k] = (int32_t)(c0 + (int64_t)(wb + q) * 32 + b);
+                ++k;
+            }
+            run += k;
+        }
+        __syncthreads();
+        for (int64_t p = s0 + threadIdx.x; p < s1; p += kBmThreads) {
+            int64_t c = colidx[p];
+            if (c >= c0 && c < c0 + kBmBits && c < K) {
+                int off = (int)(c - c0);
+                uint32_t word = bm[off >> 5];
+                rank[p] = (int32_t)(base_rank + pref[off >> 5] +
+                                    __popc(word & ((1u << (off & 31)) - 1u)));
+            }
+        }
+        base_rank += chunk_total;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        u_out[w] = (int32_t)base_rank;
+        nb_out[w] = (base_rank + kTcw - 1) / kTcw;
+    }
+}
+
+// ---------------------------------------------------------------- F2/F3
+__global__ void k_to_i32(const int64_t* __restrict__ in, int32_t* __restrict__ out, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = (int32_t)in[i];
+}
+
+// SparseAtoB: warp per window; block b's 8 columns are U[8b..8b+7], -1 padded.
+__global__ void k_fill_atob(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ rowptr,
+                            const int32_t* __restrict__ rwo, const int32_t* __restrict__ u,
+                            const int32_t* __restrict__ uniq, int32_t* __restrict__ atob) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t w = warp; w < W; w += nwarps) {
+        int64_t s0, s1;
+        window_segment(rowptr, M, nnz, w, &s0, &s1);
+        int64_t b0 = rwo[w], nb = rwo[w + 1] - b0;
+        int uw = u[w];
+        for (int64_t k = lane; k < nb * kTcw; k += 32)
+            atob[b0 * kTcw + k] = k < uw ? uniq[s0 + k] : -1;
+    }
+}
+
+// 128-bit occupancy mask per TC block: bit id set for every nnz (warp per row).
+__global__ void k_mask(int64_t M, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
+                       const int32_t* __restrict__ rank, uint32_t* __restrict__ mask) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = warp; r < M; r += nwarps) {
+        const int64_t w = r / kWindow;
+        const int lr = (int)(r % kWindow);
+        const int64_t b0 = rwo[w];
+        for (int64_t p = rowptr[r] + lane; p < rowptr[r + 1]; p += 32) {
+            int k = rank[p];
+            int64_t b = b0 + (k >> 3);
+            int id = lr * kTcw + (k & 7);
+            atomicOr(&mask[b * 4 + (id >> 5)], 1u << (id & 31));
+        }
+    }
+}
+
+__global__ void k_blkcnt(int64_t T, const uint4* __restrict__ mask, int64_t* __restrict__ cnt) {
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < T; b += (int64_t)gridDim.x * blockDim.x) {
+        uint4 m = mask[b];
+        cnt[b] = __popc(m.x) + __popc(m.y) + __popc(m.z) + __popc(m.w);
+    }
+}
+
+// Place every nnz at TCOffset[b] + (number of set ids below its id) (warp per row).
+template <class V>
+__global__ void k_place(int64_t M, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
+                        const int32_t* __restrict__ rank, const uint4* __restrict__ mask,
+                        const int32_t* __restrict__ tco, const V* __restrict__ vin,
+                        uint8_t* __restrict__ lid, V* __restrict__ vout) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = warp; r < M; r += nwarps) {
+        const int64_t w = r / kWindow;
+        const int lr = (int)(r % kWindow);
+        const int64_t b0 = rwo[w];
+        for (int64_t p = rowptr[r] + lane; p < rowptr[r + 1]; p += 32) {
+            int k = rank[p];
+            int64_t b = b0 + (k >> 3);
+            int id = lr * kTcw + (k & 7);
+            uint4 m = mask[b];
+            uint32_t words[4] = {m.x, m.y, m.z, m.w};
+            int below = 0;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                int lo = q * 32;
+                if (id >= lo + 32) below += __popc(words[q]);
+                else if (id > lo) below += __popc(words[q] & ((1u << (id - lo)) - 1u));
+            }
+            int64_t pos = (int64_t)tco[b] + below;
+            lid[pos] = (uint8_t)id;
+            vout[pos] = vin[p];
+        }
+    }
+}
+
+// ---------------------------------------------------------------- F4
+// Work units: consecutive windows whose first TC block falls in
+// the same U-block chunk form one unit; a window with more than U blocks is
+// split into ceil(nb/U) near-equal pieces (each its own unit, deterministic fixup).
+__global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, int U,
+                              int64_t* __restrict__ cnt, int64_t* __restrict__ split,
+                              int64_t* __restrict__ slots) {
+    for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
+        int64_t nb = rwo[w + 1] - rwo[w];
+        bool big = nb > U;
+        int64_t c;
+        if (big) {
+            c = (nb + U - 1) / U;
+        } else {
+            bool starts = (w == 0);
+            if (!starts) {
+                int64_t pnb = rwo[w] - rwo[w - 1];
+                starts = (pnb > U) || (rwo[w] / U != rwo[w - 1] / U);
+            }
+            c = starts ? 1 : 0;
+        }
+        cnt[w] = c;
+        split[w] = big ? 1 : 0;
+        slots[w] = big ? c : 0;
+    }
+}
+
+__global__ void k_units_fill(int64_t W, const int32_t* __restrict__ rwo, int U,
+                             const int64_t* __restrict__ ubase, const int64_t* __restrict__ sbase,
+                             const int64_t* __restrict__ slbase, Unit* __restrict__ units) {
+    for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = ubase[w + 1] - ubase[w];
+        if (c == 0) continue;
+        int64_t nb = rwo[w + 1] - rwo[w];
+        if (nb > U) {
+            for (int64_t p = 0; p < c; ++p) {
+                Unit u;
+                u.wb = (int32_t)w; u.we = (int32_t)(w + 1);
+                u.bb = (int32_t)(rwo[w] + p * nb / c);
+                u.be = (int32_t)(rwo[w] + (p + 1) * nb / c);
+                u.split_id = (int32_t)sbase[w]; u.piece = (int32_t)p; u.npieces = (int32_t)c;
+                u.slot_base = (int32_t)slbase[w];
+                units[ubase[w] + p] = u;
+            }
+        } else {
+            Unit u;
+            u.wb = (int32_t)w; u.we = -1; u.bb = rwo[w]; u.be = -1;
+            u.split_id = -1; u.piece = 0; u.npieces = 1; u.slot_base = 0;
+            units[ubase[w]] = u;
+        }
+    }
+}
+
+__global__ void k_units_fix(int64_t nu, int64_t W, const int32_t* __restrict__ rwo, Unit* __restrict__ units) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nu; i += (int64_t)gridDim.x * blockDim.x) {
+        if (units[i].split_id >= 0) continue;
+        int64_t we = (i + 1 < nu) ? units[i + 1].wb : W;
+        units[i].we = (int32_t)we;
+        units[i].be = rwo[we];
+    }
+}
+
+// ---------------------------------------------------------------- host driver
+static unsigned grid_for(int64_t work, int per_block, int cap = 1 << 20) {
+    int64_t g = (work + per_block - 1) / per_block;
+    if (g < 1) g = 1;
+    if (g > cap) g = cap;
+    return (unsigned)g;
+}
+
+static void free_format(dtc_format* h, cudaStream_t s) {
+    if (!h) return;
+    dfree(h->rwo, s); dfree(h->tco, s); dfree(h->lid, s); dfree(h->atob, s);
+    dfree(h->vals, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
+    dfree(h->stage_B, s); dfree(h->stage_C, s);
+}
+
+struct BuildTemps {
+    int* flags = nullptr;
+    int32_t* u = nullptr;
+    int64_t* nb = nullptr;       // [W+1]  -> scanned in place to block offsets
+    int32_t* uniq = nullptr;     // [nnz]
+    int32_t* rank = nullptr;     // [nnz]
+    int64_t* scan_tmp = nullptr;
+    uint32_t* mask = nullptr;    // [4T]
+    int64_t* cnt = nullptr;      // [T+1]
+    int64_t* ucnt = nullptr;     // [W+1]
+    int64_t* usplit = nullptr;   // [W+1]
+    int64_t* uslots = nullptr;   // [W+1]
+    int64_t* host = nullptr;     // pinned readback
+    void release(cudaStream_t s) {
+        dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s);
+        dfree(scan_tmp, s); dfree(mask, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
+        dfree(uslots, s);
+        if (host) cudaFreeHost(host);
+        host = nullptr;
+    }
+};
+
+static int auto_unit_blocks(int64_t T) {
+    int64_t target = T / ((int64_t)num_sms() * 16);
+    if (target < 8) target = 8;
+    if (target > 256) target = 256;
+    return (int)target;
+}
+
+int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s, dtc_format** out) {
+    if (!out) { set_error("out is NULL"); return DTC_ERR_INVALID; }
+    *out = nullptr;
+    if (!csr) { set_error("csr is NULL"); return DTC_ERR_INVALID; }
+    const int64_t M = csr->M, K = csr->K, nnz = csr->nnz;
+    if (M < 0 || K < 0 || nnz < 0 || nnz >= INT32_MAX || M >= INT32_MAX - 16 || K >= INT32_MAX) {
+        set_error("bad sizes M=%lld K=%lld nnz=%lld", (long long)M, (long long)K, (long long)nnz);
+        return DTC_ERR_INVALID;
+    }
+    if (csr->dtype != DTC_TF32 && csr->dtype != DTC_FP16) { set_error("bad dtype %d", csr->dtype); return DTC_ERR_INVALID; }
+    if (!csr->rowptr || (nnz > 0 && (!csr->colidx || !csr->vals))) { set_error("null CSR pointer"); return DTC_ERR_INVALID; }
+    if (M == 0 && nnz != 0) { set_error("M == 0 but nnz != 0"); return DTC_ERR_INVALID; }
+    int dev_count = 0;
+    if (cudaGetDeviceCount(&dev_count) != cudaSuccess || dev_count == 0) {
+        cudaGetLastError();
+        set_error("no CUDA device");
+        return DTC_ERR_CUDA;
+    }
+    const int mode = opts ? opts->dedup_path : 0;
+    const int64_t W = (M + kWindow - 1) / kWindow;
+
+    dtc_format* h = new (std::nothrow) dtc_format();
+    if (!h) { set_error("host OOM"); return DTC_ERR_OOM; }
+    h->M = M; h->K = K; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
+    cudaGetDevice(&h->device);
+    BuildTemps t;
+    int rc = DTC_OK;
+#define TRY(x) do { rc = (x); if (rc != DTC_OK) goto fail; } while (0)
+#define TRYC(x) do { cudaError_t _e = (x); if (_e != cudaSuccess) { rc = cuda_fail(_e, #x, __FILE__, __LINE__); goto fail; } } while (0)
+    {
+        TRYC(cudaMallocHost((void**)&t.host, 8 * sizeof(int64_t)));
+        TRY(dalloc(&t.flags, 1, s));
+        TRYC(cudaMemsetAsync(t.flags, 0, sizeof(int), s));
+        TRY(dalloc(&t.u, W + 1, s));
+        TRY(dalloc(&t.nb, W + 1, s));
+        TRY(dalloc(&t.uniq, nnz, s));
+        TRY(dalloc(&t.rank, nnz, s));
+        const int64_t scan_n = std::max<int64_t>(W + 1, 1);
+        // F0
+        if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, t.flags);
+        // F1
+        if (W > 0) {
+            k_dedup_sort<<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, mode,
+                                                             t.u, t.nb, t.uniq, t.rank);
+            const size_t bm_smem = 2 * kBmWords * sizeof(uint32_t);
+            TRYC(cudaFuncSetAttribute(k_dedup_bitmap, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+            k_dedup_bitmap<<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, mode,
+                                                                   t.u, t.nb, t.uniq, t.rank);
+        }
+        TRYC(cudaGetLastError());
+        // F2: RowWindowOffset = exclusive scan of nTC_w
+        TRY(dalloc(&t.scan_tmp, scan_tmp_elems(scan_n) + 64, s));
+        if (W > 0) exclusive_scan_i64(t.nb, t.nb, W, t.scan_tmp, s);
+        else TRYC(cudaMemsetAsync(t.nb, 0, sizeof(int64_t), s));
+        TRYC(cudaMemcpyAsync(&t.host[0], t.nb + W, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        TRYC(cudaMemcpyAsync(&t.host[1], t.flags, sizeof(int), cudaMemcpyDeviceToHost, s));
+        TRYC(cudaStreamSynchronize(s));  // host sync #1: T and the validation flag
+        const int64_t T = t.host[0];
+        const int flags = (int)(t.host[1] & 0xffffffff);
+        if (flags) {
+            if (flags & F_INVALID) { set_error("malformed rowptr"); rc = DTC_ERR_INVALID; }
+            else if (flags & F_RANGE) { set_error("column index out of [0, K)"); rc = DTC_ERR_RANGE; }
+            else if (flags & F_DUPLICATE) { set_error("duplicate column within a row"); rc = DTC_ERR_DUPLICATE; }
+            else { set_error("columns not ascending within a row"); rc = DTC_ERR_UNSORTED; }
+            goto fail;
+        }
+        if (T >= INT32_MAX / 8) { set_error("NumTCBlock %lld too large for int32 indexing", (long long)T); rc = DTC_ERR_UNSUPPORTED; goto fail; }
+        h->T = T;
+        // F3
+        TRY(dalloc(&h->rwo, W + 1, s));
+        TRY(dalloc(&h->tco, T + 1, s));
+        TRY(dalloc(&h->lid, nnz, s));
+        TRY(dalloc(&h->atob, 8 * T, s));
+        TRYC(cudaMallocAsync(&h->vals, std::max<int64_t>(nnz, 1) * elt_size(h->dtype), s));
+        k_to_i32<<<grid_for(W + 1, 256, 4096), 256, 0, s>>>(t.nb, h->rwo, W + 1);
+        if (T > 0) {
+            k_fill_atob<<<grid_for(W * 32, 256, 148 * 64), 256, 0, s>>>(W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, h->atob);
+            TRY(dalloc(&t.mask, 4 * T, s));
+            TRYC(cudaMemsetAsync(t.mask, 0, 4 * T * sizeof(uint32_t), s));
+            k_mask<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, csr->rowptr, h->rwo, t.rank, t.mask);
+            TRY(dalloc(&t.cnt, T + 1, s));
+            k_blkcnt<<<grid_for(T, 256, 148 * 64), 256, 0, s>>>(T, (const uint4*)t.mask, t.cnt);
+            dfree(t.scan_tmp, s);
+            TRY(dalloc(&t.scan_tmp, scan_tmp_elems(T + 1) + 64, s));
+            exclusive_scan_i64(t.cnt, t.cnt, T, t.scan_tmp, s);
+            k_to_i32<<<grid_for(T + 1, 256, 148 * 64), 256, 0, s>>>(t.cnt, h->tco, T + 1);
+            if (h->dtype == DTC_FP16)
+                k_place<uint16_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
+                    M, csr->rowptr, h->rwo, t.rank, (const uint4*)t.mask, h->tco,
+                    (const uint16_t*)csr->vals, h->lid, (uint16_t*)h->vals);
+            else
+                k_place<uint32_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
+                    M, csr->rowptr, h->rwo, t.rank, (const uint4*)t.mask, h->tco,
+                    (const uint32_t*)csr->vals, h->lid, (uint32_t*)h->vals);
+        } else {
+            TRYC(cudaMemsetAsync(h->tco, 0, sizeof(int32_t), s));
+        }
+        TRYC(cudaGetLastError());
+        // F4: work units
+        int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T);
+        h->unit_blocks = U;
+        if (W > 0) {
+            TRY(dalloc(&t.ucnt, W + 1, s));
+            TRY(dalloc(&t.usplit, W + 1, s));
+            TRY(dalloc(&t.uslots, W + 1, s));
+            k_units_count<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, U, t.ucnt, t.usplit, t.uslots);
+            dfree(t.scan_tmp, s);
+            TRY(dalloc(&t.scan_tmp, scan_tmp_elems(W + 1) + 64, s));
+            exclusive_scan_i64(t.ucnt, t.ucnt, W, t.scan_tmp, s);
+            exclusive_scan_i64(t.usplit, t.usplit, W, t.scan_tmp, s);
+            exclusive_scan_i64(t.uslots, t.uslots, W, t.scan_tmp, s);
+            TRYC(cudaMemcpyAsync(&t.host[2], t.ucnt + W, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            TRYC(cudaMemcpyAsync(&t.host[3], t.usplit + W, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            TRYC(cudaMemcpyAsync(&t.host[4], t.uslots + W, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            TRYC(cudaStreamSynchronize(s));  // host sync #2: unit count
+            h->num_units = t.host[2];
+            h->num_split = t.host[3];
+            h->num_slots = t.host[4];
+            TRY(dalloc(&h->units, std::max<int64_t>(h->num_units, 1), s));
+            k_units_fill<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, U, t.ucnt, t.usplit, t.uslots, h->units);
+            k_units_fix<<<grid_for(h->num_units, 256, 4096), 256, 0, s>>>(h->num_units, W, h->rwo, h->units);
+        }
+        TRYC(cudaGetLastError());
+        t.release(s);
+        TRYC(cudaStreamSynchronize(s));
+        *out = h;
+        return DTC_OK;
+    }
+fail:
+    cudaGetLastError();
+    t.release(s);
+    free_format(h, s);
+    cudaStreamSynchronize(s);
+    delete h;
+    return rc;
+#undef TRY
+#undef TRYC
+}
+
+}  // namespace dtc
+
+using namespace dtc;
+
+extern "C" int dtc_format_build_ex(const dtc_csr_t* csr, const dtc_build_opts_t* opts, void* stream,
+                                   dtc_handle_t* out) {
+    return format_build(csr, opts, (cudaStream_t)stream, out);
+}
+
+extern "C" int dtc_format_build(const dtc_csr_t* csr, void* stream, dtc_handle_t* out) {
+    return format_build(csr, nullptr, (cudaStream_t)stream, out);
+}
+
+extern "C" int dtc_format_query(dtc_handle_t h, dtc_format_view_t* v) {
+    if (!h || !v) { set_error("null handle or view"); return DTC_ERR_INVALID; }
+    v->M = h->M; v->K = h->K; v->nnz = h->nnz; v->num_windows = h->W; v->num_tc_blocks = h->T;
+    v->num_units = h->num_units; v->num_split_windows = h->num_split;
+    v->dtype = h->dtype; v->unit_blocks = h->unit_blocks;
+    v->row_window_offset = h->rwo; v->tc_offset = h->tco; v->tc_local_id = h->lid;
+    v->sparse_a_to_b = h->atob; v->tc_values = h->vals; v->units = (const int32_t*)h->units;
+    return DTC_OK;
+}
+
+extern "C" int dtc_format_export(dtc_handle_t h, int32_t* rwo, int32_t* tco, uint8_t* lid, int32_t* atob,
+                                 void* vals, int32_t* units) {
+    if (!h) { set_error("null handle"); return DTC_ERR_INVALID; }
+    DTC_CUDA(cudaDeviceSynchronize());
+    if (rwo) DTC_CUDA(cudaMemcpy(rwo, h->rwo, (h->W + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (tco) DTC_CUDA(cudaMemcpy(tco, h->tco, (h->T + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (lid && h->nnz) DTC_CUDA(cudaMemcpy(lid, h->lid, h->nnz, cudaMemcpyDeviceToHost));
+    if (atob && h->T) DTC_CUDA(cudaMemcpy(atob, h->atob, 8 * h->T * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (vals && h->nnz) DTC_CUDA(cudaMemcpy(vals, h->vals, h->nnz * elt_size(h->dtype), cudaMemcpyDeviceToHost));
+    if (units && h->num_units) DTC_CUDA(cudaMemcpy(units, h->units, h->num_units * sizeof(Unit), cudaMemcpyDeviceToHost));
+    return DTC_OK;
+}
+
+extern "C" void dtc_format_destroy(dtc_handle_t h) {
+    if (!h) return;
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(h->device);
+    cudaDeviceSynchronize();
+    free_format(h, 0);
+    cudaDeviceSynchronize();
+    cudaSetDevice(prev);
+    delete h;
+}

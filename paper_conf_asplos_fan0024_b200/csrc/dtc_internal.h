@@ -1,0 +1,105 @@
+// dtc_internal.h -- private declarations shared by the libdtc.so translation units.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstdio>
+#include <string>
+
+#include "../../include/dtc.h"
+
+namespace dtc {
+
+constexpr int kWindow = 16;   // BLOCK_HEIGHT
+constexpr int kTcw = 8;       // TC block width
+
+// Work-unit record (F4).  Unit u covers TC blocks [bb, be) and the C rows of
+// windows [wb, we).  split_id >= 0 marks one piece of a window that was split
+// across several units: its partial goes to workspace slot (slot_base + piece)
+// and the last arriving piece sums slots in order (deterministic fixup).
+struct Unit {
+    int32_t wb, we, bb, be;
+    int32_t split_id, piece, npieces, slot_base;
+};
+static_assert(sizeof(Unit) == 32, "unit record is 8 x int32");
+
+}  // namespace dtc
+
+struct dtc_format {
+    int64_t M = 0, K = 0, nnz = 0, W = 0, T = 0;
+    int32_t dtype = 0;
+    int32_t unit_blocks = 0;
+    int device = 0;
+    int32_t* rwo = nullptr;      // [W+1]
+    int32_t* tco = nullptr;      // [T+1]
+    uint8_t* lid = nullptr;      // [nnz]
+    int32_t* atob = nullptr;     // [8T]
+    void* vals = nullptr;        // [nnz] fp32 / fp16
+    // F4 schedule
+    int64_t num_units = 0;
+    int64_t num_split = 0;       // split windows
+    int64_t num_slots = 0;       // total split pieces
+    dtc::Unit* units = nullptr;
+    // split fixup state: counters [num_split * max_colgroups], workspace (grows with N)
+    int32_t* counters = nullptr;
+    int64_t counters_len = 0;
+    float* ws = nullptr;
+    size_t ws_bytes = 0;
+    // host-API staging buffers
+    void* stage_B = nullptr;
+    size_t stage_B_bytes = 0;
+    float* stage_C = nullptr;
+    size_t stage_C_bytes = 0;
+};
+
+namespace dtc {
+
+// thread-local last error
+void set_error(const char* fmt, ...);
+int cuda_fail(cudaError_t e, const char* what, const char* file, int line);
+
+#define DTC_CUDA(call)                                                            \
+    do {                                                                          \
+        cudaError_t _e = (call);                                                  \
+        if (_e != cudaSuccess) return ::dtc::cuda_fail(_e, #call, __FILE__, __LINE__); \
+    } while (0)
+
+// device-wide exclusive scan of n int64 values (in != out allowed, in-place
+// allowed); out[n] receives the total.  tmp must hold scan_tmp_elems(n).
+int64_t scan_tmp_elems(int64_t n);
+void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* tmp,
+                        cudaStream_t s);
+
+inline int elt_size(int32_t dtype) { return dtype == DTC_FP16 ? 2 : 4; }
+
+// stream-ordered device allocation helpers (cudaMallocAsync pool)
+template <class T>
+int dalloc(T** p, size_t count, cudaStream_t s) {
+    *p = nullptr;
+    if (count == 0) count = 1;
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(p), count * sizeof(T), s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("device allocation of %zu bytes failed: %s", count * sizeof(T),
+                  cudaGetErrorString(e));
+        return DTC_ERR_OOM;
+    }
+    return DTC_OK;
+}
+template <class T>
+void dfree(T*& p, cudaStream_t s) {
+    if (p) cudaFreeAsync(reinterpret_cast<void*>(p), s);
+    p = nullptr;
+}
+
+int num_sms();
+
+// SpMM kernel launcher (dtc_spmm.cu)
+int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc,
+                cudaStream_t s);
+
+// internal build used by the distributed layer: optional row range of the csr
+int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s,
+                 dtc_format** out);
+
+}  // namespace dtc

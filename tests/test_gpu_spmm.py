@@ -1,0 +1,215 @@
+"""S1-S5 (dtc_spmm) on the GPU vs oracle O1, through the C ABI.
+
+Tolerance |dC| <= rtol*(|A|.|B|) + 1e-6 with rtol 2e-3 (TF32) / 1e-2 (FP16)
+(BASELINE.json north_star); bit-exact where the arithmetic is exact (P2-P5).
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from datagen import configs
+
+from gpu_util import build, dev, spmm, check_tol
+
+pytestmark = pytest.mark.gpu
+
+
+def _torch():
+    import torch
+    return torch
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("N", [1, 3, 8, 32, 33, 64, 100, 128, 256, 512])
+def test_random_tolerance(dtype, N):
+    M, K = 700, 900
+    rp, ci = datagen.random_csr(M, K, 0.03, N)
+    v = datagen.uniform(N, 1, len(ci))
+    B = datagen.uniform(N, 2, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    C = spmm(f, B)
+    check_tol(C, M, K, rp, ci, v, B, dtype)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("name,N", [("c1", 32), ("c2", 128), ("c1", 256)])
+def test_p2_integer_bit_exact(name, N, dtype):
+    """P2: |a|,|b| <= 4 integers: exact in TF32/FP16 and in FP32 accumulation."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.integers(cfg.seed_a, 5, len(ci))
+    B = datagen.integers(cfg.seed_b, 6, cfg.K * N).reshape(cfg.K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype)
+    C = spmm(f, B)
+    Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v.astype(np.float32), B.astype(np.float32))
+    assert np.array_equal(C.astype(np.float64), Cr)
+
+
+def test_p3_identity_and_p4_permutation():
+    M, N = 1000, 64
+    B = datagen.uniform(1, 2, M * N).reshape(M, N)
+    Bt = B.view(np.uint32) & np.uint32(0xFFFFE000)   # pre-rounded to TF32 by truncation...
+    Bt = Bt.view(np.float32)                        # ...so RN(tf32) is the identity on it
+    rp = np.arange(M + 1, dtype=np.int32)
+    f = build(M, M, rp, np.arange(M, dtype=np.int32), np.ones(M, np.float32))
+    assert np.array_equal(spmm(f, Bt), Bt)
+    perm = np.random.default_rng(1).permutation(M).astype(np.int32)
+    # A = P stored as canonical CSR: row i has the single column perm[i]
+    f = build(M, M, rp, perm, np.ones(M, np.float32))
+    assert np.array_equal(spmm(f, Bt), Bt[perm])
+
+
+def test_p5_row_sums():
+    cfg = configs.get("c2")
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.dyadic(3, 1, len(ci), -1, 1)
+    N = 16
+    f = build(cfg.M, cfg.K, rp, ci, v)
+    C = spmm(f, np.ones((cfg.K, N), np.float32))
+    rows = np.repeat(np.arange(cfg.M), np.diff(rp))
+    sums = np.zeros(cfg.M)
+    np.add.at(sums, rows, v.astype(np.float64))
+    for j in range(N):
+        assert np.array_equal(C[:, j].astype(np.float64), sums)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+def test_p6_column_independence(dtype):
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = datagen.uniform(3, 2, cfg.K * 64).reshape(cfg.K, 64)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype)
+    C64 = spmm(f, B)
+    for j in (0, 5, 63):
+        C1 = spmm(f, np.ascontiguousarray(B[:, j:j + 1]))
+        assert np.array_equal(C1[:, 0], C64[:, j])
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("U", [1, 2, 5])
+def test_split_windows_fixup(U, dtype):
+    """Tiny work units force many split windows: the deterministic fixup path."""
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    N = 96
+    B = datagen.uniform(4, 2, cfg.K * N).reshape(cfg.K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U)
+    assert f.num_split_windows > 0
+    C1 = spmm(f, B)
+    C2 = spmm(f, B)
+    assert np.array_equal(C1, C2)                     # deterministic, counters self-reset
+    check_tol(C1, cfg.M, cfg.K, rp, ci, v, B, dtype)
+
+
+def test_deterministic_and_overwrites_everything():
+    torch = _torch()
+    cfg = configs.get("c2")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    N = 128
+    B = dev(configs.make_B(cfg, N))
+    f = build(cfg.M, cfg.K, rp, ci, v)
+    C1 = torch.full((cfg.M, N), float("nan"), device="cuda")
+    f.spmm(B, C1)
+    C2 = torch.full((cfg.M, N), float("nan"), device="cuda")
+    f.spmm(B, C2)
+    torch.cuda.synchronize()
+    assert not torch.isnan(C1).any()
+    assert torch.equal(C1, C2)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+def test_strided_and_misaligned_scalar_path(dtype):
+    torch = _torch()
+    M, K, N = 300, 400, 37
+    rp, ci = datagen.random_csr(M, K, 0.05, 7)
+    v = datagen.uniform(7, 1, len(ci))
+    Bf = datagen.uniform(7, 2, K * 50).reshape(K, 50)
+    if dtype == "fp16":
+        v, Bf = v.astype(np.float16), Bf.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    Bd = dev(Bf)[:, 1:1 + N]             # ldb = 50, misaligned start
+    Cbig = torch.full((M, 41), float("nan"), device="cuda")
+    C = Cbig[:, 2:2 + N]                 # ldc = 41, misaligned
+    f.spmm(Bd, C)
+    torch.cuda.synchronize()
+    check_tol(C.cpu().numpy(), M, K, rp, ci, v, Bf[:, 1:1 + N], dtype)
+    assert torch.isnan(Cbig[:, :2]).all() and torch.isnan(Cbig[:, 2 + N:]).all()
+
+
+def test_empty_and_tail_windows():
+    M, K, N = 37, 20, 8
+    rows = {0: [1, 2], 36: [19]}
+    rp = np.zeros(M + 1, np.int32)
+    ci = []
+    for i in range(M):
+        ci += rows.get(i, [])
+        rp[i + 1] = len(ci)
+    ci = np.array(ci, np.int32)
+    v = np.array([1.0, 2.0, 3.0], np.float32)
+    B = datagen.integers(1, 2, K * N).reshape(K, N)
+    f = build(M, K, rp, ci, v)
+    C = spmm(f, B)
+    Cr, _ = oracle.spmm(M, K, rp, ci, v, B)
+    assert np.array_equal(C.astype(np.float64), Cr)
+    # all-zero matrix
+    f0 = build(M, K, np.zeros(M + 1, np.int32), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    assert np.all(spmm(f0, B) == 0)
+
+
+def test_host_api_matches_device():
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg)
+    f = build(cfg.M, cfg.K, rp, ci, v)
+    C1 = spmm(f, B)
+    C2 = f.spmm_host(B)
+    assert np.array_equal(C1, C2)
+
+
+def _sample(cfg, rp, rng, n=4096):
+    """Sampled (row, col) pairs: uniform rows plus every row of the heaviest window."""
+    rows = rng.integers(0, cfg.M, size=n)
+    deg = np.diff(rp)
+    w = np.argmax(np.add.reduceat(deg, np.arange(0, cfg.M, 16)))
+    hub = np.arange(16 * w, min(16 * w + 16, cfg.M))
+    rows = np.concatenate([rows, np.repeat(hub, 8), [cfg.M - 1] * 8])
+    return rows.astype(np.int64)
+
+
+@pytest.mark.parametrize("name,N", [("c1", 32), ("c2", 128), ("c3", 256), ("c3h", 256),
+                                    ("c4", 64), ("c4", 128), ("c4", 256), ("c5", 512)])
+def test_config_full_size(name, N):
+    """Every BASELINE config at full size in the bench launch configuration:
+    c1/c2 compared element by element, the large ones on sampled outputs."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg, N)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=cfg.dtype)
+    C = spmm(f, B)
+    assert np.isfinite(C).all()
+    if cfg.M * N <= 50_000_000:
+        check_tol(C, cfg.M, cfg.K, rp, ci, v, B, cfg.dtype)
+        return
+    rng = np.random.default_rng(0)
+    rows = _sample(cfg, rp, rng)
+    cols = rng.integers(0, N, size=len(rows)).astype(np.int64)
+    Cr, Bd = oracle.spmm_at(cfg.M, rp, ci, v.astype(np.float32), B.astype(np.float32), rows, cols)
+    ok, ratio = oracle.within_tolerance(C[rows, cols], Cr, Bd, oracle.TOL[cfg.dtype])
+    assert ok, ratio
+    # all columns of a few whole rows, including the last (tail window) row
+    for r0 in (0, cfg.M - 3):
+        check_tol(C[r0:r0 + 3], cfg.M, cfg.K, rp, ci, v, B, cfg.dtype, r0=r0, r1=r0 + 3)
