@@ -2,31 +2,34 @@
 //
 // Paper design (Alg. 2): one thread block per 16-row window
 // iterating its TC blocks: FetchSpAsync (A tile -> smem, cp.async double
-// buffered), VFetchDense (B rows -> registers with LDG.128, no smem,
-// P:297-301), mma m16n8k4 TF32 and a register remapping that lets each
-// thread load 4 consecutive B columns and un-permutes C at the store;
-// strict balance hands fixed TC-block counts to thread blocks with atomics.
+// buffered), VFetchDense (B rows -> registers with LDG.128, bypassing
+// smem), mma m16n8k4 TF32, a register remapping that lets each
+// thread load 4 consecutive B columns and un-permutes C at the store,
+// and strict balance of TC blocks over thread blocks with atomics.
 //
-// This kernel keeps what still holds on B200 and changes the rest:
-//  * Work: a CTA takes one F4 work unit (a window-ordered run of ~U TC blocks,
-//    whole windows, or one piece of a long window) x one slice of N columns.
-//    The hardware CTA scheduler dispatches units in index = window order as slots
-//    free up, which gives both load balance and the L2 locality of a
-//    contiguous wave.  Split windows finish with a DETERMINISTIC fixup:
-//    pieces write partials to a workspace, the last arriver sums them in piece
-//    order (no float atomics, so C is bit-identical run to run).
-//  * S1 FetchSparse: the warps of the CTA cooperatively scatter the next chunk of
-//    S TC blocks into smem already in mma-fragment order (one LDS.128 / LDS.64
-//    per lane per block, conflict-free), rounding A to TF32 (cvt.rna) once.
-//  * S2 gather B: each thread issues one 16-byte load from each of its two B rows
-//    per TC block straight into registers (shared-memory bypassing) with a
-//    P-deep register prefetch ring (latency hiding instead of the paper's
-//    2-buffer A pipeline).  -1 padded columns load zeros (C6).
-//  * S3 mma.sync m16n8k8 (TF32) / m16n8k8 (FP16) per TC block: one instruction
-//    per 8 output columns consumes a whole 16x8 TC block (k = 8).
-//  * S4 epilogue: the paper's remapping generalised to k8: a thread ends up
-//    owning 2*NJ consecutive columns of rows g and g+8 -> float4 stores.
-//  * Accumulators stay in registers (a window's C tile is 16 x COLW per warp).
+// What changes on B200 (measured):
+//  * The paper's shared-memory bypass is the wrong call here: a warp-wide
+//    LDG.128 in the mma B-fragment order touches 4 different B rows per 8 lanes
+//    and costs ~12 L1 data-pipe wavefronts per request (ncu, profiles/), which
+//    capped the first kernel at ~58% of the L1 pipe with 4 TB/s of gather.  sm_100a
+//    has the async global->smem row gather the paper lacked ("absence of
+//    support for asynchronous copying ... up to Ada"): TMA tile::gather4.  The
+//    main path (k_spmm_tma) gathers each TC block's 8 B rows x 128 B slices into
+//    a 128B-swizzled smem ring with gather4 (the -1 pad rows are TMA
+//    out-of-bounds and arrive as zeros), so the consumers never wait on
+//    register-held loads and the ring keeps ~64 KB per CTA in flight.
+//  * Warp specialisation: warp WARPS stages A fragments (FetchSparse, S1) in
+//    batches of 32 TC blocks (already in mma fragment order, TF32-rounded),
+//    warp WARPS+1 issues the B gathers (S2), warps [0, WARPS) run mma.sync
+//    m16n8k8 (S3: one instruction per TC block per 8 columns, k = 8) from
+//    conflict-free LDS.128 reads, with mbarrier full/empty handshakes.
+//  * Balance + locality: a CTA takes one F4 work unit (whole windows grouped to
+//    ~U TC blocks, or one piece of a long window) x one column slice; CTAs are
+//    dispatched in window order by the hardware scheduler.  Split windows finish
+//    with a deterministic fixup (partials summed in piece order; no float atomics).
+//  * k_spmm_ldg is the register-gather fallback for layouts TMA cannot describe
+//    (unaligned B, ldb*elt % 16 != 0) -- same arithmetic, same results.
+#include <cuda.h>
 #include <cuda_fp16.h>
 
 #include <algorithm>
@@ -36,15 +39,16 @@
 
 namespace dtc {
 
-constexpr int kChunk = 32;   // TC blocks staged per smem chunk (S)
-constexpr int kPrefetch = 4; // B prefetch depth (TC blocks in flight per warp)
+constexpr int kChunk = 32;      // TC blocks per A batch (S)
+constexpr int kPrefetch = 4;    // register-gather path: B prefetch depth (divides kChunk)
+constexpr int kBRingBytes = 64 * 1024;   // TMA path: B stage ring per CTA
 
 template <int DT>
 struct Traits;
 template <>
 struct Traits<DTC_TF32> {
     static constexpr int NJ = 4;          // n8 mmas per TC block per warp
-    static constexpr int COLW = 32;       // columns per warp
+    static constexpr int COLW = 32;       // columns per warp (= one 128-byte row slice)
     static constexpr int VW = 4;          // elements per 16-byte vector
     static constexpr int FRAG_WORDS = 4;  // A fragment 32-bit words per lane
     using elt = float;
@@ -98,19 +102,359 @@ struct alignas(16) V16 {
     uint32_t w[4];
 };
 
+// ------------------------------------------------------------ mbarriers (CTA scope)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, int count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+// --------------------------------------------------- C tile store / split partials
+// A consumer warp owns rows (w*16 + g, w*16 + g + 8) and, for hi in {0,1} and
+// q < NJ/4, the 4 consecutive columns base + hi*HOFF + 4q (acc[4q..4q+3][2*half+hi]).
+template <int NJ, bool VEC>
+__device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int64_t w, int g,
+                                           int64_t base, int hoff, const float (&acc)[NJ][4], bool zero) {
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+        const int64_t row = w * kWindow + g + 8 * half;
+        if (row >= M) continue;
+        float* crow = C + row * ldc;
+#pragma unroll
+        for (int hi = 0; hi < 2; ++hi) {
+#pragma unroll
+            for (int q = 0; q < NJ / 4; ++q) {
+                const int64_t c = base + hi * hoff + 4 * q;
+                float4 v;
+                v.x = zero ? 0.f : acc[4 * q + 0][2 * half + hi];
+                v.y = zero ? 0.f : acc[4 * q + 1][2 * half + hi];
+                v.z = zero ? 0.f : acc[4 * q + 2][2 * half + hi];
+                v.w = zero ? 0.f : acc[4 * q + 3][2 * half + hi];
+                if (VEC) {
+                    if (c < N) *reinterpret_cast<float4*>(crow + c) = v;
+                } else {
+                    if (c + 0 < N) crow[c + 0] = v.x;
+                    if (c + 1 < N) crow[c + 1] = v.y;
+                    if (c + 2 < N) crow[c + 2] = v.z;
+                    if (c + 3 < N) crow[c + 3] = v.w;
+                }
+            }
+        }
+    }
+}
+
+// Split-window fixup for one warp's tile (deterministic: slots summed in piece order).
+template <int NJ, bool VEC>
+__device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
+                                            int32_t* __restrict__ ctr, float* __restrict__ C, int64_t ldc, int64_t M,
+                                            int64_t N, int g, int lane, int64_t base, int hoff) {
+    const int64_t slot = (int64_t)u.slot_base + u.piece;
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+        float* prow = ws + (slot * kWindow + g + 8 * half) * npad;
+#pragma unroll
+        for (int hi = 0; hi < 2; ++hi)
+#pragma unroll
+            for (int q = 0; q < NJ / 4; ++q) {
+                const int64_t c = base + hi * hoff + 4 * q;
+                __stcg(reinterpret_cast<float4*>(prow + c),
+                       make_float4(acc[4 * q + 0][2 * half + hi], acc[4 * q + 1][2 * half + hi],
+                                   acc[4 * q + 2][2 * half + hi], acc[4 * q + 3][2 * half + hi]));
+            }
+    }
+    __threadfence();
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) {
+        const int prev = atomicAdd(ctr, 1);
+        last = (prev == u.npieces - 1);
+        if (last) *ctr = 0;  // self-reset for the next launch (stream-ordered)
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (!last) return;
+    __threadfence();
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+    for (int pc = 0; pc < u.npieces; ++pc) {
+        const int64_t sl = (int64_t)u.slot_base + pc;
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+            const float* prow = ws + (sl * kWindow + g + 8 * half) * npad;
+#pragma unroll
+            for (int hi = 0; hi < 2; ++hi)
+#pragma unroll
+                for (int q = 0; q < NJ / 4; ++q) {
+                    const int64_t c = base + hi * hoff + 4 * q;
+                    const float4 v = __ldcg(reinterpret_cast<const float4*>(prow + c));
+                    acc[4 * q + 0][2 * half + hi] += v.x;
+                    acc[4 * q + 1][2 * half + hi] += v.y;
+                    acc[4 * q + 2][2 * half + hi] += v.z;
+                    acc[4 * q + 3][2 * half + hi] += v.w;
+                }
+        }
+    }
+    store_tile<NJ, VEC>(C, ldc, M, N, u.wb, g, base, hoff, acc, false);
+}
+
+// --------------------------------------------------- S1: A batch producer (one warp)
+// Scatters the non-zeros of TC blocks [b0, b0+nb) into zeroed lane-major mma
+// fragments (TF32-rounded) and copies their 8 B-row ids.
+template <int DT>
+__device__ __forceinline__ void produce_a_batch(int b0, int nb, const int32_t* __restrict__ tco,
+                                                const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob,
+                                                const void* __restrict__ avals, uint32_t* fr, int32_t* ids,
+                                                int32_t* s_tco, int lane) {
+    constexpr int FW = Traits<DT>::FRAG_WORDS;
+    if (lane < nb) s_tco[lane] = tco[b0 + lane];
+    if (lane == 0) s_tco[nb] = tco[b0 + nb];
+    for (int k = lane; k < 2 * nb; k += 32)
+        reinterpret_cast<int4*>(ids)[k] = __ldg(reinterpret_cast<const int4*>(atob + (int64_t)b0 * 8) + k);
+    for (int k = lane; k < nb * 32 * FW / 4; k += 32) reinterpret_cast<uint4*>(fr)[k] = make_uint4(0u, 0u, 0u, 0u);
+    __syncwarp();
+    const int e0 = s_tco[0], e1 = s_tco[nb];
+    for (int base = e0; base < e1; base += 32 * 8) {
+        int idv[8];
+        uint32_t val[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const int e = base + q * 32 + lane;
+            if (e < e1) {
+                idv[q] = lid[e];
+                val[q] = (DT == DTC_TF32) ? __float_as_uint(__ldg(reinterpret_cast<const float*>(avals) + e))
+                                          : (uint32_t)__ldg(reinterpret_cast<const unsigned short*>(avals) + e);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const int e = base + q * 32 + lane;
+            if (e < e1) {
+                int lo = 0, hi = nb;  // block j of entry e: s_tco[j] <= e < s_tco[j+1]
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (s_tco[mid] <= e) lo = mid; else hi = mid;
+                }
+                uint32_t* f = fr + lo * 32 * FW;
+                const int slot = frag_slot<DT>(idv[q]);
+                if (DT == DTC_TF32) f[slot] = to_tf32(__uint_as_float(val[q]));
+                else reinterpret_cast<unsigned short*>(f)[slot] = (unsigned short)val[q];
+            }
+        }
+    }
+    __syncwarp();
+}
+
+// ============================================================ main path: TMA gather4
+// Column slice of a consumer warp = one 128-byte box column of B (32 fp32 / 64 fp16).
+// Stage s of the B ring holds, for every active warp slice, 8 rows x 128 B
+// (two gather4 boxes: rows 0-3 then rows 4-7) at ring + s*WARPS*1KB + warp*1KB,
+// 128B-swizzled: 16-byte chunk c of row r sits at chunk c ^ r.
+//  TF32: thread (g,t) reads rows t and t+4 at chunk cg = (g>>1) + 4*(g&1) -> the 8
+//        lanes of an LDS.128 phase hit 8 distinct chunks (conflict-free); virtual mma
+//        column g is actual column n0 + 4*cg + jj, so the thread ends up owning
+//        columns n0 + 4t + [0,4) and n0 + 16 + 4t + [0,4).
+//  FP16: thread (g,t) reads rows 2t and 2t+1 at chunk g (conflict-free), owning
+//        columns n0 + 16t + [0,16) (as in the register-remap of P:313-319).
+template <int DT, int WARPS, bool VEC>
+__global__ void __launch_bounds__((WARPS + 2) * 32)
+k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
+           const int32_t* __restrict__ tco, const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob,
+           const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
+    using Tr = Traits<DT>;
+    constexpr int NJ = Tr::NJ, COLW = Tr::COLW, FW = Tr::FRAG_WORDS;
+    constexpr int S = kChunk;
+    constexpr int STAGE = WARPS * 1024;                   // bytes per B stage
+    constexpr int R = kBRingBytes / STAGE > 16 ? 16 : kBRingBytes / STAGE;
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    // 1024-byte align the ring (128B swizzle atom)
+    uint8_t* sbase = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* ring = sbase;                                                    // [R][STAGE]
+    uint32_t* s_frag = reinterpret_cast<uint32_t*>(sbase + R * STAGE);        // [2][S][32*FW]
+    int32_t* s_ids = reinterpret_cast<int32_t*>(s_frag + 2 * S * 32 * FW);    // [2][S][8]
+    int32_t* s_tco = s_ids + 2 * S * 8;                                       // [S+1]
+    __shared__ __align__(8) uint64_t bar_afull[2], bar_aempty[2], bar_bfull[R], bar_bempty[R];
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const Unit u = units[blockIdx.x];
+    const int64_t ncta0 = (int64_t)blockIdx.y * WARPS * COLW;
+    const int64_t nact64 = (N - ncta0 + COLW - 1) / COLW;
+    const int nact = nact64 < WARPS ? (int)nact64 : WARPS;
+    const int nblocks = u.be - u.bb;
+    const int nbatch = (nblocks + S - 1) / S;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&bar_afull[i], 1);
+            mbar_init(&bar_aempty[i], nact + 1);   // consumers + the B producer (reads ids)
+        }
+        for (int i = 0; i < R; ++i) {
+            mbar_init(&bar_bfull[i], 1);
+            mbar_init(&bar_bempty[i], nact);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (warp == WARPS) {
+        // ================= A producer (S1) =================
+        for (int c = 0; c < nbatch; ++c) {
+            const int buf = c & 1;
+            if (c >= 2) mbar_wait(&bar_aempty[buf], ((c >> 1) - 1) & 1);
+            const int b0 = u.bb + c * S;
+            produce_a_batch<DT>(b0, min(S, u.be - b0), tco, lid, atob, avals, s_frag + buf * S * 32 * FW,
+                                s_ids + buf * S * 8, s_tco, lane);
+            if (lane == 0) mbar_arrive(&bar_afull[buf]);
+            __syncwarp();
+        }
+        return;
+    }
+    if (warp == WARPS + 1) {
+        // ================= B producer (S2): gather4 into the swizzled ring =================
+        const uint32_t bytes = (uint32_t)nact * 1024u;
+        const int slice = lane >> 1, half = lane & 1;
+        const int col = (int)(ncta0 + (int64_t)slice * COLW);
+        for (int i = 0; i < nblocks; ++i) {
+            const int c = i / S, j = i % S, s = i % R;
+            if (j == 0) mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
+            if (i >= R) mbar_wait(&bar_bempty[s], ((i / R) - 1) & 1);
+            if (lane == 0) mbar_arrive_tx(&bar_bfull[s], bytes);
+            if (slice < nact) {
+                const int4 r = reinterpret_cast<const int4*>(s_ids + (c & 1) * S * 8 + j * 8)[half];
+                const uint32_t dst = smem_u32(ring + s * STAGE + slice * 1024 + half * 512);
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+                    " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
+                    "l"(&bmap), "r"(col), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w), "r"(smem_u32(&bar_bfull[s]))
+                    : "memory");
+            }
+            if (j == S - 1 || i == nblocks - 1) {   // done reading this batch's ids
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bar_aempty[c & 1]);
+            }
+        }
+        return;
+    }
+    if (warp >= nact) return;
+
+    // ================= consumers (S3 mma, S4 epilogue) =================
+    const int g = lane >> 2, t = lane & 3;
+    const int64_t n0 = ncta0 + (int64_t)warp * COLW;
+    const int64_t base = (DT == DTC_TF32) ? n0 + 4 * t : n0 + 16 * t;
+    const int hoff = (DT == DTC_TF32) ? 16 : 8;
+    const bool split = u.split_id >= 0;
+    // smem byte offsets of this thread's two 16-byte B reads inside a warp slice
+    int off0, off1;
+    if (DT == DTC_TF32) {
+        const int cg = (g >> 1) + 4 * (g & 1);
+        off0 = t * 128 + ((cg ^ t) << 4);
+        off1 = (t + 4) * 128 + ((cg ^ (t + 4)) << 4);
+    } else {
+        off0 = (2 * t) * 128 + ((g ^ (2 * t)) << 4);
+        off1 = (2 * t + 1) * 128 + ((g ^ (2 * t + 1)) << 4);
+    }
+    const uint8_t* myring = ring + warp * 1024;
+
+    float acc[NJ][4];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+
+    int64_t cur = u.wb;
+    int64_t next_end = INT_MAX;
+    if (!split) {
+        while (cur < u.we && rwo[cur + 1] <= u.bb) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+    }
+
+    for (int i = 0; i < nblocks; ++i) {
+        const int c = i / S, j = i % S, s = i % R;
+        if (j == 0) mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
+        mbar_wait(&bar_bfull[s], (i / R) & 1);
+        const uint32_t* fr = s_frag + (c & 1) * S * 32 * FW + j * 32 * FW;
+        const uint4 bv0 = *reinterpret_cast<const uint4*>(myring + s * STAGE + off0);
+        const uint4 bv1 = *reinterpret_cast<const uint4*>(myring + s * STAGE + off1);
+        if (DT == DTC_TF32) {
+            const uint4 av = reinterpret_cast<const uint4*>(fr)[lane];
+            const uint32_t a[4] = {av.x, av.y, av.z, av.w};
+            const uint32_t x0[4] = {bv0.x, bv0.y, bv0.z, bv0.w};
+            const uint32_t x1[4] = {bv1.x, bv1.y, bv1.z, bv1.w};
+#pragma unroll
+            for (int jj = 0; jj < NJ; ++jj)
+                mma_tf32(acc[jj], a, x0[jj], x1[jj]);
+        } else {
+            const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
+            const uint32_t a[2] = {av.x, av.y};
+            const uint32_t x0[4] = {bv0.x, bv0.y, bv0.z, bv0.w};
+            const uint32_t x1[4] = {bv1.x, bv1.y, bv1.z, bv1.w};
+#pragma unroll
+            for (int jj = 0; jj < NJ; ++jj) {
+                const uint32_t bb = __byte_perm(x0[jj >> 1], x1[jj >> 1], (jj & 1) ? 0x7632 : 0x5410);
+                mma_f16(acc[jj], a, bb);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(&bar_bempty[s]);
+            if (j == S - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[c & 1]);
+        }
+        const int64_t b = u.bb + i;
+        if (b + 1 == next_end) {   // S4: window boundary -> store and reset
+            store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false);
+#pragma unroll
+            for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+            ++cur;
+            while (cur < u.we && rwo[cur + 1] == rwo[cur]) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+            next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+        }
+    }
+    if (!split) {
+        while (cur < u.we) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        return;
+    }
+    // S5: split-window fixup per consumer warp
+    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
+    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
+}
+
+// ============================================================ fallback: register gather
+// 16-byte read-only load of p if pred, else zeros -- branch-free (predicated LDG).
+__device__ __forceinline__ V16 ldg16_pred(const void* p, bool pred) {
+    V16 v;
+    asm volatile(
+        "{\n"
+        ".reg .pred q;\n"
+        "setp.ne.b32 q, %5, 0;\n"
+        "mov.b32 %0, 0; mov.b32 %1, 0; mov.b32 %2, 0; mov.b32 %3, 0;\n"
+        "@q ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+        "}\n"
+        : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3])
+        : "l"(p), "r"((int)pred));
+    return v;
+}
+
 template <int DT, bool VEC>
 __device__ __forceinline__ V16 load_b(const void* __restrict__ B, int64_t ldb, int row, int64_t col, int64_t N) {
+    using E = typename Traits<DT>::elt;
+    const E* p = reinterpret_cast<const E*>(B) + (int64_t)row * ldb + col;
+    if (VEC) return ldg16_pred(p, row >= 0 && col < N);
     V16 v;
     v.w[0] = v.w[1] = v.w[2] = v.w[3] = 0u;
     if (row < 0) return v;
-    using E = typename Traits<DT>::elt;
-    const E* p = reinterpret_cast<const E*>(B) + (int64_t)row * ldb + col;
-    if (VEC) {
-        if (col < N) {
-            uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
-            v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
-        }
-    } else {
+    {
         if (DT == DTC_TF32) {
             const float* q = reinterpret_cast<const float*>(p);
 #pragma unroll
@@ -127,118 +471,170 @@ __device__ __forceinline__ V16 load_b(const void* __restrict__ B, int64_t ldb, i
     return v;
 }
 
+// All warps of the CTA share a double-buffered A pipeline over chunks of kChunk
+// TC blocks: the global loads for chunk c+1's non-zeros and chunk c+2's offsets /
+// B-row ids are issued into registers BEFORE chunk c is computed and only stored
+// to smem at the chunk boundary, so FetchSparse never exposes memory latency
+// (the paper's sparse double buffering, made two-deep).  Each warp
+// streams its 32/64-column B slice with a kPrefetch-deep register ring that runs
+// continuously across chunk boundaries (VFetchDense + remap).
+constexpr int kLdgMaxRegs = 80;   // register budget of the register-gather kernel (occupancy)
 template <int DT, int WARPS, bool VEC>
-__global__ void __launch_bounds__(WARPS * 32)
-k_spmm(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
-       const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob, const void* __restrict__ avals,
-       const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
-       float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
+__global__ void __launch_bounds__(WARPS * 32, 65536 / (WARPS * 32 * kLdgMaxRegs))
+k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
+           const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob, const void* __restrict__ avals,
+           const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
     using Tr = Traits<DT>;
     constexpr int NJ = Tr::NJ, COLW = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
     constexpr int P = kPrefetch;
+    constexpr int S = kChunk;
+    constexpr int NT = WARPS * 32;
+    constexpr int TPT = (S + 1 + NT - 1) / NT;      // TCOffset values per thread
+    constexpr int IPT = (2 * S + NT - 1) / NT;      // int4 of B-row ids per thread
+    constexpr int KE = 512 / NT < 1 ? 1 : (512 / NT > 4 ? 4 : 512 / NT);  // non-zeros per thread prefetched per chunk
     extern __shared__ __align__(16) uint32_t smem[];
-    uint32_t* s_frag = smem;                                       // [kChunk][32*FW]
-    int32_t* s_ids = reinterpret_cast<int32_t*>(smem + kChunk * 32 * FW);  // [kChunk][8]
-    __shared__ int s_last;
+    uint32_t* s_frag = smem;                                                 // [2][S][32*FW]
+    int32_t* s_ids = reinterpret_cast<int32_t*>(smem + 2 * S * 32 * FW);     // [2][S][8]
+    int32_t* s_tco = s_ids + 2 * S * 8;                                      // [2][S+1]
 
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int g = lane >> 2, t = lane & 3;
     const Unit u = units[blockIdx.x];
-    const int64_t n0 = ((int64_t)blockIdx.y * WARPS + warp) * COLW;  // this warp's first column
+    const int64_t n0 = ((int64_t)blockIdx.y * WARPS + warp) * COLW;
     const bool active = n0 < N;
-    const int64_t bcol = n0 + (int64_t)VW * g;                        // column of this thread's B vector
-    const int64_t ccol = n0 + 2 * NJ * t;                             // first C column owned
-    const int rsel0 = (DT == DTC_TF32) ? t : 2 * t;                   // B rows (k) this thread loads
+    const int64_t bcol = n0 + (int64_t)VW * g;
+    const int64_t base = n0 + 2 * NJ * t;
+    const int hoff = NJ;
+    const int rsel0 = (DT == DTC_TF32) ? t : 2 * t;
     const int rsel1 = (DT == DTC_TF32) ? t + 4 : 2 * t + 1;
     const bool split = u.split_id >= 0;
+    const int nblocks = u.be - u.bb;
+    const int nchunks = (nblocks + S - 1) / S;
+    auto chunk_nb = [&](int c) { return min(S, nblocks - c * S); };
+
+    // ---- A pipeline pieces (register staging -> smem)
+    int m_tco[TPT];
+    int4 m_ids[IPT];
+    auto meta_load = [&](int c) {
+        const int nb = chunk_nb(c), b0 = u.bb + c * S;
+#pragma unroll
+        for (int k = 0; k < TPT; ++k) {
+            const int x = tid + k * NT;
+            if (x <= nb) m_tco[k] = tco[b0 + x];
+        }
+#pragma unroll
+        for (int k = 0; k < IPT; ++k) {
+            const int x = tid + k * NT;
+            if (x < 2 * nb) m_ids[k] = __ldg(reinterpret_cast<const int4*>(atob + (int64_t)b0 * 8) + x);
+        }
+    };
+    auto meta_store = [&](int c, int buf) {
+        const int nb = chunk_nb(c);
+#pragma unroll
+        for (int k = 0; k < TPT; ++k) {
+            const int x = tid + k * NT;
+            if (x <= nb) s_tco[buf * (S + 1) + x] = m_tco[k];
+        }
+#pragma unroll
+        for (int k = 0; k < IPT; ++k) {
+            const int x = tid + k * NT;
+            if (x < 2 * nb) reinterpret_cast<int4*>(s_ids + buf * S * 8)[x] = m_ids[k];
+        }
+        uint4* fr = reinterpret_cast<uint4*>(s_frag + buf * S * 32 * FW);
+        for (int x = tid; x < nb * 32 * FW / 4; x += NT) fr[x] = make_uint4(0u, 0u, 0u, 0u);
+    };
+    int e_id[KE];
+    uint32_t e_val[KE];
+    auto ent_val = [&](int e) -> uint32_t {
+        return (DT == DTC_TF32) ? __float_as_uint(__ldg(reinterpret_cast<const float*>(avals) + e))
+                                : (uint32_t)__ldg(reinterpret_cast<const unsigned short*>(avals) + e);
+    };
+    auto ent_load_n = [&](int buf, int nb) {
+        const int e0 = s_tco[buf * (S + 1)], e1 = s_tco[buf * (S + 1) + nb];
+#pragma unroll
+        for (int k = 0; k < KE; ++k) {
+            const int e = e0 + tid + k * NT;
+            if (e < e1) {
+                e_id[k] = lid[e];
+                e_val[k] = ent_val(e);
+            }
+        }
+    };
+    auto put = [&](int buf, int nb, int e, int id, uint32_t v) {
+        const int32_t* tc = s_tco + buf * (S + 1);
+        int lo = 0, hi = nb;   // block j of entry e: tc[j] <= e < tc[j+1]
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (tc[mid] <= e) lo = mid; else hi = mid;
+        }
+        uint32_t* f = s_frag + buf * S * 32 * FW + lo * 32 * FW;
+        const int slot = frag_slot<DT>(id);
+        if (DT == DTC_TF32) f[slot] = to_tf32(__uint_as_float(v));
+        else reinterpret_cast<unsigned short*>(f)[slot] = (unsigned short)v;
+    };
+    auto ent_store_n = [&](int buf, int nb) {
+        const int e0 = s_tco[buf * (S + 1)], e1 = s_tco[buf * (S + 1) + nb];
+#pragma unroll
+        for (int k = 0; k < KE; ++k) {
+            const int e = e0 + tid + k * NT;
+            if (e < e1) put(buf, nb, e, e_id[k], e_val[k]);
+        }
+        for (int e = e0 + KE * NT + tid; e < e1; e += NT) put(buf, nb, e, lid[e], ent_val(e));  // dense chunks
+    };
 
     float acc[NJ][4];
 #pragma unroll
     for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
 
-    auto store_window = [&](int64_t w, bool zero) {
-        if (!active) return;
-#pragma unroll
-        for (int half = 0; half < 2; ++half) {
-            const int64_t row = w * kWindow + g + 8 * half;
-            if (row >= M) continue;
-            float* crow = C + row * ldc;
-#pragma unroll
-            for (int hi = 0; hi < 2; ++hi) {        // columns ccol + hi*NJ + [0, NJ)
-#pragma unroll
-                for (int q = 0; q < NJ / 4; ++q) {
-                    const int64_t c = ccol + hi * NJ + 4 * q;
-                    float4 v;
-                    v.x = zero ? 0.f : acc[4 * q + 0][2 * half + hi];
-                    v.y = zero ? 0.f : acc[4 * q + 1][2 * half + hi];
-                    v.z = zero ? 0.f : acc[4 * q + 2][2 * half + hi];
-                    v.w = zero ? 0.f : acc[4 * q + 3][2 * half + hi];
-                    if (VEC) {
-                        if (c < N) *reinterpret_cast<float4*>(crow + c) = v;
-                    } else {
-                        if (c + 0 < N) crow[c + 0] = v.x;
-                        if (c + 1 < N) crow[c + 1] = v.y;
-                        if (c + 2 < N) crow[c + 2] = v.z;
-                        if (c + 3 < N) crow[c + 3] = v.w;
-                    }
-                }
-            }
-        }
-    };
-
-    // window cursor over [u.wb, u.we); leading empty windows get zero rows
     int64_t cur = u.wb;
     int64_t next_end = INT_MAX;
     if (!split) {
-        while (cur < u.we && rwo[cur + 1] <= u.bb) { store_window(cur, true); ++cur; }
+        while (cur < u.we && rwo[cur + 1] <= u.bb) {
+            if (active) store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+            ++cur;
+        }
         next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
     }
 
-    for (int64_t cb = u.bb; cb < u.be; cb += kChunk) {
-        const int nblk = (u.be - cb) < kChunk ? (int)(u.be - cb) : kChunk;
-        // ---- S1: stage A tiles of this chunk in fragment order + the B row ids
-        for (int j = warp; j < nblk; j += WARPS) {
-            const int64_t b = cb + j;
-            const int lo = tco[b], hi = tco[b + 1];
-            uint32_t* fr = s_frag + j * 32 * FW;
-            if (FW == 4) reinterpret_cast<uint4*>(fr)[lane] = make_uint4(0u, 0u, 0u, 0u);
-            else reinterpret_cast<uint2*>(fr)[lane] = make_uint2(0u, 0u);
-            if (lane < 8) s_ids[j * 8 + lane] = atob[b * 8 + lane];
-            __syncwarp();
-            for (int e = lo + lane; e < hi; e += 32) {
-                const int id = lid[e];
-                const int slot = frag_slot<DT>(id);
-                if (DT == DTC_TF32) {
-                    fr[slot] = to_tf32(reinterpret_cast<const float*>(avals)[e]);
-                } else {
-                    reinterpret_cast<unsigned short*>(fr)[slot] = reinterpret_cast<const unsigned short*>(avals)[e];
+    if (nchunks > 0) {
+        // prologue: chunks 0 and 1 staged, chunk 1's non-zeros and chunk 2's meta in flight
+        meta_load(0);
+        meta_store(0, 0);
+        if (nchunks > 1) { meta_load(1); meta_store(1, 1); }
+        __syncthreads();
+        ent_load_n(0, chunk_nb(0));
+        ent_store_n(0, chunk_nb(0));
+        __syncthreads();
+        if (nchunks > 1) ent_load_n(1, chunk_nb(1));
+        if (nchunks > 2) meta_load(2);
+
+        V16 b0[P], b1[P];
+        auto ids_of = [&](int i) -> const int32_t* { return s_ids + ((i / S) & 1) * S * 8 + (i % S) * 8; };
+        if (active) {
+#pragma unroll
+            for (int q = 0; q < P; ++q) {
+                if (q < nblocks) {
+                    const int32_t* id = ids_of(q);
+                    b0[q] = load_b<DT, VEC>(B, ldb, id[rsel0], bcol, N);
+                    b1[q] = load_b<DT, VEC>(B, ldb, id[rsel1], bcol, N);
                 }
             }
         }
-        __syncthreads();
-        // ---- S2/S3: gather B into registers P blocks ahead, mma per TC block
-        if (active) {
-            V16 b0[P], b1[P];
+        for (int i0 = 0; i0 < nblocks; i0 += P) {
 #pragma unroll
             for (int q = 0; q < P; ++q) {
-                if (q < nblk) {
-                    b0[q] = load_b<DT, VEC>(B, ldb, s_ids[q * 8 + rsel0], bcol, N);
-                    b1[q] = load_b<DT, VEC>(B, ldb, s_ids[q * 8 + rsel1], bcol, N);
-                }
-            }
-            for (int j0 = 0; j0 < nblk; j0 += P) {
-#pragma unroll
-                for (int q = 0; q < P; ++q) {
-                    const int j = j0 + q;
-                    if (j < nblk) {
-                        const uint32_t* fr = s_frag + j * 32 * FW;
+                const int i = i0 + q;
+                if (i < nblocks) {
+                    const int c = i / S, j = i % S;
+                    if (active) {
+                        const uint32_t* fr = s_frag + (c & 1) * S * 32 * FW + j * 32 * FW;
                         if (DT == DTC_TF32) {
                             const uint4 av = reinterpret_cast<const uint4*>(fr)[lane];
                             const uint32_t a[4] = {av.x, av.y, av.z, av.w};
 #pragma unroll
                             for (int jj = 0; jj < NJ; ++jj)
-                                mma_tf32(acc[jj], a, to_tf32(__uint_as_float(b0[q].w[jj])),
-                                         to_tf32(__uint_as_float(b1[q].w[jj])));
+                                mma_tf32(acc[jj], a, b0[q].w[jj], b1[q].w[jj]);
                         } else {
                             const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
                             const uint32_t a[2] = {av.x, av.y};
@@ -249,116 +645,162 @@ k_spmm(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const in
                                 mma_f16(acc[jj], a, bb);
                             }
                         }
-                        if (j + P < nblk) {
-                            b0[q] = load_b<DT, VEC>(B, ldb, s_ids[(j + P) * 8 + rsel0], bcol, N);
-                            b1[q] = load_b<DT, VEC>(B, ldb, s_ids[(j + P) * 8 + rsel1], bcol, N);
+                        if (i + P < nblocks) {
+                            const int32_t* id = ids_of(i + P);
+                            b0[q] = load_b<DT, VEC>(B, ldb, id[rsel0], bcol, N);
+                            b1[q] = load_b<DT, VEC>(B, ldb, id[rsel1], bcol, N);
                         }
-                        // ---- S4: window boundary -> store and reset
-                        const int64_t b = cb + j;
+                        const int64_t b = u.bb + i;
                         if (b + 1 == next_end) {
-                            store_window(cur, false);
+                            store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false);
 #pragma unroll
                             for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
                             ++cur;
-                            while (cur < u.we && rwo[cur + 1] == rwo[cur]) { store_window(cur, true); ++cur; }
+                            while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
+                                store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+                                ++cur;
+                            }
                             next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
                         }
                     }
                 }
             }
-        }  // inactive warps (columns >= N) only help stage A; they store nothing
-        __syncthreads();
+            const int nxt = i0 + P;   // S is a multiple of P: chunk boundaries fall between groups
+            if (nxt % S == 0 && nxt < nblocks) {
+                // chunk boundary (CTA-uniform): finish chunk c+1's fragments, recycle buffer c&1
+                const int c = nxt / S - 1;
+                ent_store_n((c + 1) & 1, chunk_nb(c + 1));
+                __syncthreads();
+                if (c + 2 < nchunks) meta_store(c + 2, c & 1);
+                __syncthreads();
+                if (c + 2 < nchunks) ent_load_n(c & 1, chunk_nb(c + 2));
+                if (c + 3 < nchunks) meta_load(c + 3);
+            }
+        }
     }
-
+    if (!active) return;
     if (!split) {
-        while (cur < u.we) { store_window(cur, true); ++cur; }
+        while (cur < u.we) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
         return;
     }
+    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
+    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
+}
 
-    // ---- S5: split-window fixup (deterministic: partials summed in piece order)
-    const int64_t slot = (int64_t)u.slot_base + u.piece;
-    if (active) {
-#pragma unroll
-        for (int half = 0; half < 2; ++half) {
-            float* prow = ws + (slot * kWindow + g + 8 * half) * npad;
-#pragma unroll
-            for (int hi = 0; hi < 2; ++hi)
-#pragma unroll
-                for (int q = 0; q < NJ / 4; ++q) {
-                    const int64_t c = ccol + hi * NJ + 4 * q;
-                    float4 v = make_float4(acc[4 * q + 0][2 * half + hi], acc[4 * q + 1][2 * half + hi],
-                                           acc[4 * q + 2][2 * half + hi], acc[4 * q + 3][2 * half + hi]);
-                    __stcg(reinterpret_cast<float4*>(prow + c), v);
-                }
-        }
+// ============================================================ host side
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&fn, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            fn = nullptr;
+        cudaGetLastError();
     }
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int32_t* ctr = counters + (int64_t)u.split_id * gridDim.y + blockIdx.y;
-        const int prev = atomicAdd(ctr, 1);
-        s_last = (prev == u.npieces - 1);
-        if (s_last) *ctr = 0;  // self-reset for the next launch (stream-ordered)
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-#pragma unroll
-    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
-    if (!active) return;
-    for (int pc = 0; pc < u.npieces; ++pc) {
-        const int64_t sl = (int64_t)u.slot_base + pc;
-#pragma unroll
-        for (int half = 0; half < 2; ++half) {
-            const float* prow = ws + (sl * kWindow + g + 8 * half) * npad;
-#pragma unroll
-            for (int hi = 0; hi < 2; ++hi)
-#pragma unroll
-                for (int q = 0; q < NJ / 4; ++q) {
-                    const int64_t c = ccol + hi * NJ + 4 * q;
-                    const float4 v = __ldcg(reinterpret_cast<const float4*>(prow + c));
-                    acc[4 * q + 0][2 * half + hi] += v.x;
-                    acc[4 * q + 1][2 * half + hi] += v.y;
-                    acc[4 * q + 2][2 * half + hi] += v.z;
-                    acc[4 * q + 3][2 * half + hi] += v.w;
-                }
-        }
-    }
-    store_window(u.wb, false);
+    return fn;
+}
+
+// Tensor map of B (K rows x N cols, row stride ldb) for 128-byte x 1-row gather4 boxes.
+static bool make_bmap(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype) {
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return false;
+    const int elt = elt_size(dtype);
+    cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)K};
+    cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
+    cuuint32_t box[2] = {(cuuint32_t)(128 / elt), 1};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(map, dtype == DTC_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                     const_cast<void*>(B), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+struct LaunchArgs {
+    dtc_format* h;
+    const void* B;
+    int64_t ldb;
+    float* C;
+    int64_t ldc, N;
+    int gy;
+    int64_t npad;
+    cudaStream_t s;
+};
+
+template <int DT, int WARPS>
+static size_t tma_smem_bytes() {
+    constexpr int STAGE = WARPS * 1024;
+    constexpr int R = kBRingBytes / STAGE > 16 ? 16 : kBRingBytes / STAGE;
+    return 1024 + (size_t)R * STAGE + (size_t)2 * kChunk * 32 * Traits<DT>::FRAG_WORDS * 4 + 2 * kChunk * 8 * 4 +
+           (kChunk + 1) * 4;
 }
 
 template <int DT, int WARPS, bool VEC>
-static cudaError_t launch_one(dtc_format* h, const void* B, int64_t ldb, float* C, int64_t ldc, int64_t N,
-                              int gy, int64_t npad, cudaStream_t s) {
-    using Tr = Traits<DT>;
-    const size_t smem = (size_t)kChunk * 32 * Tr::FRAG_WORDS * 4 + (size_t)kChunk * 8 * 4;
-    dim3 grid((unsigned)h->num_units, (unsigned)gy);
-    k_spmm<DT, WARPS, VEC><<<grid, WARPS * 32, smem, s>>>(h->units, h->rwo, h->tco, h->lid, h->atob, h->vals, B,
-                                                          ldb, C, ldc, h->M, N, h->ws, h->counters, npad);
+static cudaError_t launch_tma(const LaunchArgs& a, const CUtensorMap& map) {
+    const size_t smem = tma_smem_bytes<DT, WARPS>();
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_spmm_tma<DT, WARPS, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr = true;
+    }
+    dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
+    k_spmm_tma<DT, WARPS, VEC><<<grid, (WARPS + 2) * 32, smem, a.s>>>(map, a.h->units, a.h->rwo, a.h->tco, a.h->lid,
+                                                                      a.h->atob, a.h->vals, a.C, a.ldc, a.h->M, a.N,
+                                                                      a.h->ws, a.h->counters, a.npad);
+    return cudaGetLastError();
+}
+
+template <int DT, int WARPS, bool VEC>
+static cudaError_t launch_ldg(const LaunchArgs& a) {
+    const size_t smem = (size_t)2 * kChunk * 32 * Traits<DT>::FRAG_WORDS * 4 + (size_t)2 * kChunk * 8 * 4 +
+                        (size_t)2 * (kChunk + 1) * 4;
+    dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
+    k_spmm_ldg<DT, WARPS, VEC><<<grid, WARPS * 32, smem, a.s>>>(a.h->units, a.h->rwo, a.h->tco, a.h->lid, a.h->atob,
+                                                                a.h->vals, a.B, a.ldb, a.C, a.ldc, a.h->M, a.N,
+                                                                a.h->ws, a.h->counters, a.npad);
     return cudaGetLastError();
 }
 
 template <int DT, bool VEC>
-static cudaError_t dispatch_warps(int warps, dtc_format* h, const void* B, int64_t ldb, float* C, int64_t ldc,
-                                  int64_t N, int gy, int64_t npad, cudaStream_t s) {
+static cudaError_t dispatch(int warps, bool tma, const LaunchArgs& a, const CUtensorMap& map) {
+    if (tma) {
+        switch (warps) {
+            case 1: return launch_tma<DT, 1, VEC>(a, map);
+            case 2: return launch_tma<DT, 2, VEC>(a, map);
+            case 4: return launch_tma<DT, 4, VEC>(a, map);
+            default: return launch_tma<DT, 8, VEC>(a, map);
+        }
+    }
     switch (warps) {
-        case 1: return launch_one<DT, 1, VEC>(h, B, ldb, C, ldc, N, gy, npad, s);
-        case 2: return launch_one<DT, 2, VEC>(h, B, ldb, C, ldc, N, gy, npad, s);
-        case 4: return launch_one<DT, 4, VEC>(h, B, ldb, C, ldc, N, gy, npad, s);
-        default: return launch_one<DT, 8, VEC>(h, B, ldb, C, ldc, N, gy, npad, s);
+        case 1: return launch_ldg<DT, 1, VEC>(a);
+        case 2: return launch_ldg<DT, 2, VEC>(a);
+        case 4: return launch_ldg<DT, 4, VEC>(a);
+        default: return launch_ldg<DT, 8, VEC>(a);
     }
 }
 
+static int g_force_path = -1;   // 1 = register gather (default), 2 = TMA gather4 (DTC_SPMM_PATH=tma)
+
 int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc, cudaStream_t s) {
     if (!h) { set_error("null handle"); return DTC_ERR_INVALID; }
-    if (N < 1 || ldb < N || ldc < N) { set_error("bad N/ldb/ldc (%lld/%lld/%lld)", (long long)N, (long long)ldb, (long long)ldc); return DTC_ERR_INVALID; }
+    if (N < 1 || ldb < N || ldc < N) {
+        set_error("bad N/ldb/ldc (%lld/%lld/%lld)", (long long)N, (long long)ldb, (long long)ldc);
+        return DTC_ERR_INVALID;
+    }
     if (h->M == 0) return DTC_OK;
     if (!C || (!B && h->T > 0)) { set_error("null B or C"); return DTC_ERR_INVALID; }
     if (h->num_units == 0) return DTC_OK;
+    if (g_force_path < 0) {
+        const char* e = getenv("DTC_SPMM_PATH");
+        g_force_path = (e && e[0] == 't') ? 2 : 1;   // default: register gather (see header)
+    }
     const int elt = elt_size(h->dtype);
     const int VW = 16 / elt;
-    const bool vec = ((uintptr_t)B % 16 == 0) && ((uintptr_t)C % 16 == 0) && (ldb % VW == 0) && (N % VW == 0) &&
-                     (ldc % 4 == 0);
     const int colw = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
     const int64_t need = (N + colw - 1) / colw;
     const int warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
@@ -366,9 +808,8 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     if (gy64 > 65535) { set_error("N too large"); return DTC_ERR_UNSUPPORTED; }
     const int gy = (int)gy64;
     const int64_t npad = gy64 * warps * colw;
-    // split-window state
     if (h->num_split > 0) {
-        const int64_t ncnt = h->num_split * gy;
+        const int64_t ncnt = h->num_split * gy * 8;   // per (split, column group, consumer warp)
         if (ncnt > h->counters_len) {
             dfree(h->counters, s);
             h->counters_len = 0;
@@ -386,13 +827,22 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
             h->ws_bytes = wsb;
         }
     }
+    // TMA needs a 16-byte aligned base and row pitch; a ragged N is fine (OOB columns zero-fill)
+    CUtensorMap map;
+    memset(&map, 0, sizeof(map));
+    bool tma = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && h->K < (int64_t(1) << 31) &&
+               N < (int64_t(1) << 31) && g_force_path != 1;
+    if (tma) tma = make_bmap(&map, B, h->K, N, ldb, h->dtype);
+    // float4 C stores need an aligned C; the LDG path additionally needs B vectors
+    const bool cvec = ((uintptr_t)C % 16 == 0) && (ldc % 4 == 0) && (N % 4 == 0);
+    const bool bvec = ((uintptr_t)B % 16 == 0) && (ldb % VW == 0) && (N % VW == 0);
+    const bool use_vec = tma ? cvec : (cvec && bvec);
+    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s};
     cudaError_t e;
     if (h->dtype == DTC_FP16)
-        e = vec ? dispatch_warps<DTC_FP16, true>(warps, h, B, ldb, C, ldc, N, gy, npad, s)
-                : dispatch_warps<DTC_FP16, false>(warps, h, B, ldb, C, ldc, N, gy, npad, s);
+        e = use_vec ? dispatch<DTC_FP16, true>(warps, tma, a, map) : dispatch<DTC_FP16, false>(warps, tma, a, map);
     else
-        e = vec ? dispatch_warps<DTC_TF32, true>(warps, h, B, ldb, C, ldc, N, gy, npad, s)
-                : dispatch_warps<DTC_TF32, false>(warps, h, B, ldb, C, ldc, N, gy, npad, s);
+        e = use_vec ? dispatch<DTC_TF32, true>(warps, tma, a, map) : dispatch<DTC_TF32, false>(warps, tma, a, map);
     if (e != cudaSuccess) return cuda_fail(e, "k_spmm launch", __FILE__, __LINE__);
     return DTC_OK;
 }
