@@ -9,7 +9,7 @@ import threading
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libdtc.so")
+_SO = os.environ.get("DTC_LIBRARY") or os.path.join(_HERE, "libdtc.so")  # override: experiments only
 _HEADER = os.path.join(os.path.dirname(_HERE), "include", "dtc.h")
 
 DTC_OK = 0

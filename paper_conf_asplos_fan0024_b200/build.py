@@ -38,22 +38,23 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    if out is None and not force and not needs_build():
         return SO
+    target = out or SO
     inc, lib = nccl_paths()
     nvcc = os.environ.get("NVCC", "nvcc")
     cmd = [nvcc, "-O3", "-std=c++17", "-lineinfo", "--expt-relaxed-constexpr", *ARCH,
            "-shared", "-Xcompiler", "-fPIC", "-cudart", "static",
            "-I", os.path.join(ROOT, "include"), "-I", inc,
-           *sources(), "-o", SO + ".tmp",
+           *[f"-D{d}" for d in defines], *sources(), "-o", target + ".tmp",
            "-L", lib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + lib]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)
-    os.replace(SO + ".tmp", SO)
-    return SO
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

@@ -40,7 +40,37 @@
 namespace dtc {
 
 constexpr int kChunk = 32;      // TC blocks per A batch (S)
-constexpr int kPrefetch = 4;    // register-gather path: B prefetch depth (divides kChunk)
+// Register-gather tuning per (dtype, consumer warps): B prefetch depth P and the
+// register cap that sets occupancy (measured sweep).  The A chunk
+// is the largest multiple of P not above 32 TC blocks.  -DDTC_PREFETCH /
+// -DDTC_LDG_MAXREGS override both for sweeps.
+template <int DT, int W>
+constexpr int ldg_prefetch() {
+#ifdef DTC_PREFETCH
+    return DTC_PREFETCH;
+#else
+    return 1;
+#endif
+}
+template <int DT, int W>
+constexpr int ldg_maxregs() {
+#ifdef DTC_LDG_MAXREGS
+    return DTC_LDG_MAXREGS;
+#else
+    return 64;
+#endif
+}
+template <int DT, int W>
+constexpr int ldg_chunk_target() {
+#ifdef DTC_CHUNK
+    return DTC_CHUNK;
+#else
+    return (DT == DTC_TF32 && W <= 4) ? 16 : 32;   // smaller chunks let 8 TF32 CTAs of 4 warps fit in smem
+#endif
+}
+template <int DT, int W>
+constexpr int ldg_chunk() { return ldg_prefetch<DT, W>() * (ldg_chunk_target<DT, W>() / ldg_prefetch<DT, W>()); }
+
 constexpr int kBRingBytes = 64 * 1024;   // TMA path: B stage ring per CTA
 
 template <int DT>
@@ -431,6 +461,10 @@ k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
 }
 
 // ============================================================ fallback: register gather
+// 64 zero bytes that padded (-1) B rows and columns beyond N read instead of B
+// (branch-free gather: the address is selected, the load is unconditional).
+__device__ __align__(128) uint4 g_zero_line[8];
+
 // 16-byte read-only load of p if pred, else zeros -- branch-free (predicated LDG).
 __device__ __forceinline__ V16 ldg16_pred(const void* p, bool pred) {
     V16 v;
@@ -478,17 +512,16 @@ __device__ __forceinline__ V16 load_b(const void* __restrict__ B, int64_t ldb, i
 // (the paper's sparse double buffering, made two-deep).  Each warp
 // streams its 32/64-column B slice with a kPrefetch-deep register ring that runs
 // continuously across chunk boundaries (VFetchDense + remap).
-constexpr int kLdgMaxRegs = 80;   // register budget of the register-gather kernel (occupancy)
 template <int DT, int WARPS, bool VEC>
-__global__ void __launch_bounds__(WARPS * 32, 65536 / (WARPS * 32 * kLdgMaxRegs))
+__global__ void __launch_bounds__(WARPS * 32, (65536 / (WARPS * 32 * ldg_maxregs<DT, WARPS>())) > 32 ? 32 : (65536 / (WARPS * 32 * ldg_maxregs<DT, WARPS>())))
 k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
            const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob, const void* __restrict__ avals,
            const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
     using Tr = Traits<DT>;
     constexpr int NJ = Tr::NJ, COLW = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
-    constexpr int P = kPrefetch;
-    constexpr int S = kChunk;
+    constexpr int P = ldg_prefetch<DT, WARPS>();
+    constexpr int S = ldg_chunk<DT, WARPS>();
     constexpr int NT = WARPS * 32;
     constexpr int TPT = (S + 1 + NT - 1) / NT;      // TCOffset values per thread
     constexpr int IPT = (2 * S + NT - 1) / NT;      // int4 of B-row ids per thread
@@ -506,8 +539,6 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     const int64_t bcol = n0 + (int64_t)VW * g;
     const int64_t base = n0 + 2 * NJ * t;
     const int hoff = NJ;
-    const int rsel0 = (DT == DTC_TF32) ? t : 2 * t;
-    const int rsel1 = (DT == DTC_TF32) ? t + 4 : 2 * t + 1;
     const bool split = u.split_id >= 0;
     const int nblocks = u.be - u.bb;
     const int nchunks = (nblocks + S - 1) / S;
@@ -539,7 +570,17 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 #pragma unroll
         for (int k = 0; k < IPT; ++k) {
             const int x = tid + k * NT;
-            if (x < 2 * nb) reinterpret_cast<int4*>(s_ids + buf * S * 8)[x] = m_ids[k];
+            if (x < 2 * nb) {
+                int4 v = m_ids[k];
+                if (DT == DTC_TF32) {
+                    // block row ids r0..r7 arrive as int4 {r0..r3}, {r4..r7}; store as
+                    // r0 r4 r1 r5 r2 r6 r3 r7 so thread t reads (r_t, r_t+4) with one LDS.64
+                    int* d = s_ids + buf * S * 8 + (x >> 1) * 8 + (x & 1);
+                    d[0] = v.x; d[2] = v.y; d[4] = v.z; d[6] = v.w;
+                } else {
+                    reinterpret_cast<int4*>(s_ids + buf * S * 8)[x] = v;
+                }
+            }
         }
         uint4* fr = reinterpret_cast<uint4*>(s_frag + buf * S * 32 * FW);
         for (int x = tid; x < nb * 32 * FW / 4; x += NT) fr[x] = make_uint4(0u, 0u, 0u, 0u);
@@ -587,8 +628,8 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 #pragma unroll
     for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
 
-    int64_t cur = u.wb;
-    int64_t next_end = INT_MAX;
+    int cur = u.wb;          // window cursor (int32: W, T < 2^31)
+    int next_end = INT_MAX;
     if (!split) {
         while (cur < u.we && rwo[cur + 1] <= u.bb) {
             if (active) store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true);
@@ -610,14 +651,33 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         if (nchunks > 2) meta_load(2);
 
         V16 b0[P], b1[P];
-        auto ids_of = [&](int i) -> const int32_t* { return s_ids + ((i / S) & 1) * S * 8 + (i % S) * 8; };
+        // thread's two B rows of block i: TF32 (t, t+4), FP16 (2t, 2t+1) -> adjacent id slots 2t, 2t+1
+        auto ids_of = [&](int i) -> int2 {
+            return *reinterpret_cast<const int2*>(s_ids + ((i / S) & 1) * S * 8 + (i % S) * 8 + 2 * t);
+        };
+        // VEC: byte pointer of this thread's 16-byte column vector in B row 0; padded rows and
+        // columns >= N are redirected to the zero line (no predication, no divergence)
+        const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)sizeof(typename Tr::elt);
+        const uint64_t ldb_bytes = (uint64_t)ldb * sizeof(typename Tr::elt);
+        const bool col_ok = bcol < N;
+        auto gather = [&](int row) -> V16 {
+            if (VEC) {
+                const char* p = (row >= 0 && col_ok) ? bthr + (uint64_t)(uint32_t)row * ldb_bytes
+                                                     : reinterpret_cast<const char*>(g_zero_line);
+                const uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
+                V16 v;
+                v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
+                return v;
+            }
+            return load_b<DT, VEC>(B, ldb, row, bcol, N);
+        };
         if (active) {
 #pragma unroll
             for (int q = 0; q < P; ++q) {
                 if (q < nblocks) {
-                    const int32_t* id = ids_of(q);
-                    b0[q] = load_b<DT, VEC>(B, ldb, id[rsel0], bcol, N);
-                    b1[q] = load_b<DT, VEC>(B, ldb, id[rsel1], bcol, N);
+                    const int2 id = ids_of(q);
+                    b0[q] = gather(id.x);
+                    b1[q] = gather(id.y);
                 }
             }
         }
@@ -646,12 +706,11 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
                             }
                         }
                         if (i + P < nblocks) {
-                            const int32_t* id = ids_of(i + P);
-                            b0[q] = load_b<DT, VEC>(B, ldb, id[rsel0], bcol, N);
-                            b1[q] = load_b<DT, VEC>(B, ldb, id[rsel1], bcol, N);
+                            const int2 id = ids_of(i + P);
+                            b0[q] = gather(id.x);
+                            b1[q] = gather(id.y);
                         }
-                        const int64_t b = u.bb + i;
-                        if (b + 1 == next_end) {
+                        if (u.bb + i + 1 == next_end) {
                             store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false);
 #pragma unroll
                             for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
@@ -757,8 +816,8 @@ static cudaError_t launch_tma(const LaunchArgs& a, const CUtensorMap& map) {
 
 template <int DT, int WARPS, bool VEC>
 static cudaError_t launch_ldg(const LaunchArgs& a) {
-    const size_t smem = (size_t)2 * kChunk * 32 * Traits<DT>::FRAG_WORDS * 4 + (size_t)2 * kChunk * 8 * 4 +
-                        (size_t)2 * (kChunk + 1) * 4;
+    constexpr int S = ldg_chunk<DT, WARPS>();
+    const size_t smem = (size_t)2 * S * 32 * Traits<DT>::FRAG_WORDS * 4 + (size_t)2 * S * 8 * 4 + (size_t)2 * (S + 1) * 4;
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
     k_spmm_ldg<DT, WARPS, VEC><<<grid, WARPS * 32, smem, a.s>>>(a.h->units, a.h->rwo, a.h->tco, a.h->lid, a.h->atob,
                                                                 a.h->vals, a.B, a.ldb, a.C, a.ldc, a.h->M, a.N,
