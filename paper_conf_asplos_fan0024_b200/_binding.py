@@ -287,6 +287,14 @@ class Dist:
         _check(lib().dtc_dist_query(self._h, ctypes.byref(rb), ctypes.byref(re_), ctypes.byref(loc)),
                "dtc_dist_query")
         self.row_begin, self.row_end = rb.value, re_.value
+        self._local = loc
+
+    def local_spmm(self, B, C_local, stream=None):
+        """This rank's rows only, B already resident (no collective): C_local = A[rows] @ B."""
+        N = B.shape[1]
+        assert B.is_contiguous() and C_local.is_contiguous() and C_local.shape[0] >= self.row_end - self.row_begin
+        _check(lib().dtc_spmm(self._local, _dptr(B), N, N, _dptr(C_local), N, _stream_ptr(stream)), "dtc_spmm")
+        return C_local
 
     def spmm(self, B, C, root: int = 0, gather_c: bool = True, stream=None):
         N = B.shape[1]

@@ -110,7 +110,7 @@ extern "C" int dtc_dist_create(const dtc_csr_t* csr, int32_t rank, int32_t world
     rc = format_build(&lc, nullptr, s, &d->local);
     if (rc) { dfree(d->local_rowptr, s); cudaStreamSynchronize(s); delete d; return rc; }
     // 3. communicator
-    if (nccl_id && world > 1) {
+    if (nccl_id) {   // a 1-rank communicator is valid too (exercises the NCCL path on one GPU)
         ncclUniqueId id;
         memcpy(&id, nccl_id, sizeof(id));
         ncclResult_t nr = ncclCommInitRank(&d->comm, world, id, rank);
@@ -140,12 +140,12 @@ extern "C" int dtc_spmm_dist(dtc_dist_t d, void* B, int32_t root, int64_t N, flo
     if (d->world > 1 && !d->comm) { set_error("no communicator (created with nccl_id == NULL)"); return DTC_ERR_INVALID; }
     cudaStream_t s = (cudaStream_t)stream;
     const ncclDataType_t bt = d->dtype == DTC_FP16 ? ncclHalf : ncclFloat;
-    if (d->world > 1 && d->K > 0) DTC_NCCL(ncclBroadcast(B, B, (size_t)(d->K * N), bt, root, d->comm, s));
+    if (d->comm && d->K > 0) DTC_NCCL(ncclBroadcast(B, B, (size_t)(d->K * N), bt, root, d->comm, s));
     const int64_t r0 = d->row_begin[d->rank];
     float* Cl = gather_c ? C + r0 * N : C;
     int rc = spmm_launch(d->local, B, N, N, Cl, N, s);
     if (rc) return rc;
-    if (gather_c && d->world > 1) {
+    if (gather_c && d->comm) {
         DTC_NCCL(ncclGroupStart());
         for (int r = 0; r < d->world; ++r) {
             const int64_t a = d->row_begin[r], b = d->row_begin[r + 1];

@@ -399,10 +399,15 @@ struct BuildTemps {
     }
 };
 
-static int auto_unit_blocks(int64_t T) {
-    int64_t target = T / ((int64_t)num_sms() * 16);
-    if (target < 8) target = 8;
+// F4 unit size: ~2.5 windows' worth of TC blocks (measured sweep, DESIGN.md §5:
+// arxiv-like 32, banded 48-64, products-like 128-192, reddit-like 256), clamped to
+// [32, 256] and small enough that there are at least 2 units per SM.
+static int auto_unit_blocks(int64_t T, int64_t W) {
+    int64_t target = W > 0 ? (5 * T) / (2 * W) : 32;
+    if (target < 32) target = 32;
     if (target > 256) target = 256;
+    const int64_t cap = T / (2 * (int64_t)num_sms());
+    if (target > cap) target = cap < 8 ? 8 : cap;
     return (int)target;
 }
 
@@ -505,7 +510,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         }
         TRYC(cudaGetLastError());
         // F4: work units
-        int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T);
+        int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T, W);
         h->unit_blocks = U;
         if (W > 0) {
             TRY(dalloc(&t.ucnt, W + 1, s));
