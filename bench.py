@@ -213,11 +213,15 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
     flops = 2.0 * nnz * N
 
     if world == 1:
-        torch.cuda.synchronize()
-        tb0 = time.perf_counter()
-        fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks)
-        torch.cuda.synchronize()
-        build_ms = (time.perf_counter() - tb0) * 1e3
+        # format build (F0-F4): first call (includes one-time module/pool setup) and a warm rebuild
+        build_ms_runs = []
+        for _ in range(2):
+            torch.cuda.synchronize()
+            tb0 = time.perf_counter()
+            fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks)
+            torch.cuda.synchronize()
+            build_ms_runs.append((time.perf_counter() - tb0) * 1e3)
+        build_ms = build_ms_runs[-1]
         C_d = torch.empty((M, N), dtype=torch.float32, device=dev)
         fn = lambda: fmt.spmm(B_d, C_d)  # noqa: E731
         T = fmt.num_tc_blocks
@@ -288,6 +292,7 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
                            "kernel": "k_spmm (dtc_spmm)", "kernel_ms_mean": round(kern_ms, 5),
                            "kernel_ms_median": round(statistics.median(ms), 5)}
         out["format_build_ms"] = round(build_ms, 3)
+        out["format_build_first_call_ms"] = round(build_ms_runs[0], 3)
         out["format_build_x_spmm"] = round(build_ms / kern_ms, 2)
     out["config"] = cfgd
     out["gpu_launches"] = args.steps * dtc.launches_per_call()

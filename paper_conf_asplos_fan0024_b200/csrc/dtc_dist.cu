@@ -163,6 +163,6 @@ extern "C" void dtc_dist_destroy(dtc_dist_t d) {
     if (!d) return;
     if (d->comm) ncclCommDestroy(d->comm);
     dtc_format_destroy(d->local);
-    if (d->local_rowptr) { cudaFree(d->local_rowptr); d->local_rowptr = nullptr; }
+    if (d->local_rowptr) { dfree(d->local_rowptr, 0); cudaDeviceSynchronize(); }
     delete d;
 }

@@ -15,12 +15,13 @@
 //       k_dedup_bitmap    CTA per larger window: chunked smem bitmap over its column span
 //                         -> u_w, the window's ascending unique list, rank of every nnz
 //   F2  scan ceil(u_w/8)  -> RowWindowOffset, T                  (host sync #1)
-//   F3  k_fill_atob, k_mask (128-bit occupancy per TC block), k_blkcnt + scan ->
-//       TCOffset, k_place (position = TCOffset + popcount of lower ids)
+//   F3  k_fill_window: CTA per window -- SparseAtoB, 128-bit occupancy mask per TC block
+//       (smem atomics), TCOffset by a CTA scan, position = TCOffset + popcount of lower ids
 //   F4  k_units_count + scans + k_units_fill/fix (host sync #2: unit count)
 #include <algorithm>
 #include <climits>
 #include <cstring>
+#include <chrono>
 #include <new>
 
 #include "dtc_device.cuh"
@@ -224,79 +225,86 @@ __global__ void k_to_i32(const int64_t* __restrict__ in, int32_t* __restrict__ o
         out[i] = (int32_t)in[i];
 }
 
-// SparseAtoB: warp per window; block b's 8 columns are U[8b..8b+7], -1 padded.
-__global__ void k_fill_atob(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ rowptr,
-                            const int32_t* __restrict__ rwo, const int32_t* __restrict__ u,
-                            const int32_t* __restrict__ uniq, int32_t* __restrict__ atob) {
-    const int lane = threadIdx.x & 31;
-    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t w = warp; w < W; w += nwarps) {
-        int64_t s0, s1;
-        window_segment(rowptr, M, nnz, w, &s0, &s1);
-        int64_t b0 = rwo[w], nb = rwo[w + 1] - b0;
-        int uw = u[w];
-        for (int64_t k = lane; k < nb * kTcw; k += 32)
-            atob[b0 * kTcw + k] = k < uw ? uniq[s0 + k] : -1;
-    }
-}
+// F3, one CTA per window (no global atomics for windows of <= kFillSmemBlocks TC blocks):
+//   SparseAtoB[8*(b0+j) + i] = U[8j + i] (or -1);  a 128-bit occupancy mask per block (bit =
+//   local id) built with shared-memory atomics; TCOffset by a CTA scan of the masks' popcounts
+//   starting at rowptr[16w] (= TCOffset[RWO[w]]); every nnz then lands at
+//   TCOffset[b] + popcount(mask[b] below its id) -- ascending local id inside a block (C5).
+constexpr int kFillThreads = 256;
+constexpr int kFillSmemBlocks = 1024;
 
-// 128-bit occupancy mask per TC block: bit id set for every nnz (warp per row).
-__global__ void k_mask(int64_t M, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
-                       const int32_t* __restrict__ rank, uint32_t* __restrict__ mask) {
-    const int lane = threadIdx.x & 31;
-    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t r = warp; r < M; r += nwarps) {
-        const int64_t w = r / kWindow;
-        const int lr = (int)(r % kWindow);
-        const int64_t b0 = rwo[w];
-        for (int64_t p = rowptr[r] + lane; p < rowptr[r + 1]; p += 32) {
-            int k = rank[p];
-            int64_t b = b0 + (k >> 3);
-            int id = lr * kTcw + (k & 7);
-            atomicOr(&mask[b * 4 + (id >> 5)], 1u << (id & 31));
-        }
-    }
-}
-
-__global__ void k_blkcnt(int64_t T, const uint4* __restrict__ mask, int64_t* __restrict__ cnt) {
-    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < T; b += (int64_t)gridDim.x * blockDim.x) {
-        uint4 m = mask[b];
-        cnt[b] = __popc(m.x) + __popc(m.y) + __popc(m.z) + __popc(m.w);
-    }
-}
-
-// Place every nnz at TCOffset[b] + (number of set ids below its id) (warp per row).
 template <class V>
-__global__ void k_place(int64_t M, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
-                        const int32_t* __restrict__ rank, const uint4* __restrict__ mask,
-                        const int32_t* __restrict__ tco, const V* __restrict__ vin,
-                        uint8_t* __restrict__ lid, V* __restrict__ vout) {
-    const int lane = threadIdx.x & 31;
-    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t r = warp; r < M; r += nwarps) {
-        const int64_t w = r / kWindow;
-        const int lr = (int)(r % kWindow);
-        const int64_t b0 = rwo[w];
-        for (int64_t p = rowptr[r] + lane; p < rowptr[r + 1]; p += 32) {
-            int k = rank[p];
-            int64_t b = b0 + (k >> 3);
-            int id = lr * kTcw + (k & 7);
-            uint4 m = mask[b];
-            uint32_t words[4] = {m.x, m.y, m.z, m.w};
-            int below = 0;
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                int lo = q * 32;
-                if (id >= lo + 32) below += __popc(words[q]);
-                else if (id > lo) below += __popc(words[q] & ((1u << (id - lo)) - 1u));
-            }
-            int64_t pos = (int64_t)tco[b] + below;
-            lid[pos] = (uint8_t)id;
-            vout[pos] = vin[p];
+__global__ void __launch_bounds__(kFillThreads)
+k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
+              const int32_t* __restrict__ u, const int32_t* __restrict__ uniq, const int32_t* __restrict__ rank,
+              uint32_t* __restrict__ gmask, const V* __restrict__ vin, int32_t* __restrict__ tco,
+              uint8_t* __restrict__ lid, V* __restrict__ vout, int32_t* __restrict__ atob) {
+    __shared__ uint32_t s_mask[kFillSmemBlocks * 4];
+    __shared__ int s_off[kFillSmemBlocks];
+    __shared__ int s_rp[kWindow + 1];
+    const int tid = threadIdx.x;
+    const int64_t w = blockIdx.x;
+    int64_t s0, s1;
+    window_segment(rowptr, M, nnz, w, &s0, &s1);
+    const int64_t r0 = w * kWindow;
+    const int nrows = (M - r0) < kWindow ? (int)(M - r0) : kWindow;
+    const int64_t b0 = rwo[w];
+    const int nb = (int)(rwo[w + 1] - b0);
+    const bool sm = nb <= kFillSmemBlocks;
+    uint32_t* mask = sm ? s_mask : gmask + b0 * 4;
+    if (tid <= nrows) s_rp[tid] = (int)clamp64(rowptr[r0 + tid], s0, s1);
+    if (sm) for (int i = tid; i < nb * 4; i += kFillThreads) s_mask[i] = 0u;
+    const int uw = u[w];
+    for (int64_t k = tid; k < (int64_t)nb * kTcw; k += kFillThreads)
+        atob[b0 * kTcw + k] = k < uw ? uniq[s0 + k] : -1;
+    __syncthreads();
+    auto row_of = [&](int64_t p) {   // s_rp[r] <= p < s_rp[r+1]
+        int lo = 0, hi = nrows;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (s_rp[mid] <= p) lo = mid; else hi = mid;
         }
+        return lo;
+    };
+    for (int64_t p = s0 + tid; p < s1; p += kFillThreads) {
+        const int r = row_of(p);
+        const int k = rank[p];
+        const int id = r * kTcw + (k & 7);
+        atomicOr(&mask[(k >> 3) * 4 + (id >> 5)], 1u << (id & 31));
+    }
+    __syncthreads();
+    auto mask_word = [&](int j, int q) -> uint32_t { return sm ? s_mask[j * 4 + q] : __ldcg(mask + j * 4 + q); };
+    int64_t running = s0;
+    for (int jb = 0; jb < nb; jb += kFillThreads) {
+        const int j = jb + tid;
+        int c = 0;
+        if (j < nb) c = __popc(mask_word(j, 0)) + __popc(mask_word(j, 1)) + __popc(mask_word(j, 2)) + __popc(mask_word(j, 3));
+        int tot;
+        const int ex = block_exscan<kFillThreads>(c, &tot);
+        if (j < nb) {
+            tco[b0 + j] = (int32_t)(running + ex);
+            if (sm) s_off[j] = (int)(running + ex);
+        }
+        running += tot;
+    }
+    if (w == W - 1 && tid == 0) tco[b0 + nb] = (int32_t)nnz;
+    __syncthreads();
+    for (int64_t p = s0 + tid; p < s1; p += kFillThreads) {
+        const int r = row_of(p);
+        const int k = rank[p];
+        const int j = k >> 3;
+        const int id = r * kTcw + (k & 7);
+        int below = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int lo = q * 32;
+            const uint32_t m = mask_word(j, q);
+            if (id >= lo + 32) below += __popc(m);
+            else if (id > lo) below += __popc(m & ((1u << (id - lo)) - 1u));
+        }
+        const int64_t pos = (int64_t)(sm ? s_off[j] : __ldcg(tco + b0 + j)) + below;
+        lid[pos] = (uint8_t)id;
+        vout[pos] = vin[p];
     }
 }
 
@@ -394,8 +402,7 @@ struct BuildTemps {
         dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s);
         dfree(scan_tmp, s); dfree(mask, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
         dfree(uslots, s);
-        if (host) cudaFreeHost(host);
-        host = nullptr;
+        host = nullptr;   // per-thread pinned scratch, not owned
     }
 };
 
@@ -410,6 +417,26 @@ static int auto_unit_blocks(int64_t T, int64_t W) {
     if (target > cap) target = cap < 8 ? 8 : cap;
     return (int)target;
 }
+
+// DTC_BUILD_PROFILE=1: synchronise and print the wall time of each build stage (diagnostics only).
+struct StageTimer {
+    bool on = false;
+    cudaStream_t s = nullptr;
+    std::chrono::steady_clock::time_point t0;
+    void init(cudaStream_t st) {
+        const char* e = getenv("DTC_BUILD_PROFILE");
+        on = e && e[0] == '1';
+        s = st;
+        if (on) { cudaStreamSynchronize(s); t0 = std::chrono::steady_clock::now(); }
+    }
+    void mark(const char* what) {
+        if (!on) return;
+        cudaStreamSynchronize(s);
+        auto t1 = std::chrono::steady_clock::now();
+        fprintf(stderr, "[dtc build] %-28s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(t1 - t0).count());
+        t0 = t1;
+    }
+};
 
 int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s, dtc_format** out) {
     if (!out) { set_error("out is NULL"); return DTC_ERR_INVALID; }
@@ -437,11 +464,14 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
     h->M = M; h->K = K; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
     cudaGetDevice(&h->device);
     BuildTemps t;
+    StageTimer st;
+    st.init(s);
     int rc = DTC_OK;
 #define TRY(x) do { rc = (x); if (rc != DTC_OK) goto fail; } while (0)
 #define TRYC(x) do { cudaError_t _e = (x); if (_e != cudaSuccess) { rc = cuda_fail(_e, #x, __FILE__, __LINE__); goto fail; } } while (0)
     {
-        TRYC(cudaMallocHost((void**)&t.host, 8 * sizeof(int64_t)));
+        t.host = pinned_scratch();
+        if (!t.host) { set_error("pinned host scratch allocation failed"); rc = DTC_ERR_OOM; goto fail; }
         TRY(dalloc(&t.flags, 1, s));
         TRYC(cudaMemsetAsync(t.flags, 0, sizeof(int), s));
         TRY(dalloc(&t.u, W + 1, s));
@@ -449,8 +479,10 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         TRY(dalloc(&t.uniq, nnz, s));
         TRY(dalloc(&t.rank, nnz, s));
         const int64_t scan_n = std::max<int64_t>(W + 1, 1);
+        st.mark("setup+temp alloc");
         // F0
         if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, t.flags);
+        st.mark("F0 validate");
         // F1
         if (W > 0) {
             k_dedup_sort<<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, mode,
@@ -461,6 +493,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
                                                                    t.u, t.nb, t.uniq, t.rank);
         }
         TRYC(cudaGetLastError());
+        st.mark("F1 dedup");
         // F2: RowWindowOffset = exclusive scan of nTC_w
         TRY(dalloc(&t.scan_tmp, scan_tmp_elems(scan_n) + 64, s));
         if (W > 0) exclusive_scan_i64(t.nb, t.nb, W, t.scan_tmp, s);
@@ -479,36 +512,35 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         }
         if (T >= INT32_MAX / 8) { set_error("NumTCBlock %lld too large for int32 indexing", (long long)T); rc = DTC_ERR_UNSUPPORTED; goto fail; }
         h->T = T;
+        st.mark("F2 scan+sync");
         // F3
         TRY(dalloc(&h->rwo, W + 1, s));
         TRY(dalloc(&h->tco, T + 1, s));
         TRY(dalloc(&h->lid, nnz, s));
         TRY(dalloc(&h->atob, 8 * T, s));
-        TRYC(cudaMallocAsync(&h->vals, std::max<int64_t>(nnz, 1) * elt_size(h->dtype), s));
+        {
+            uint8_t* vb = nullptr;
+            TRY(dalloc(&vb, (size_t)std::max<int64_t>(nnz, 1) * elt_size(h->dtype), s));
+            h->vals = vb;
+        }
         k_to_i32<<<grid_for(W + 1, 256, 4096), 256, 0, s>>>(t.nb, h->rwo, W + 1);
         if (T > 0) {
-            k_fill_atob<<<grid_for(W * 32, 256, 148 * 64), 256, 0, s>>>(W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, h->atob);
+            // global mask words only back windows with more than kFillSmemBlocks TC blocks
             TRY(dalloc(&t.mask, 4 * T, s));
             TRYC(cudaMemsetAsync(t.mask, 0, 4 * T * sizeof(uint32_t), s));
-            k_mask<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, csr->rowptr, h->rwo, t.rank, t.mask);
-            TRY(dalloc(&t.cnt, T + 1, s));
-            k_blkcnt<<<grid_for(T, 256, 148 * 64), 256, 0, s>>>(T, (const uint4*)t.mask, t.cnt);
-            dfree(t.scan_tmp, s);
-            TRY(dalloc(&t.scan_tmp, scan_tmp_elems(T + 1) + 64, s));
-            exclusive_scan_i64(t.cnt, t.cnt, T, t.scan_tmp, s);
-            k_to_i32<<<grid_for(T + 1, 256, 148 * 64), 256, 0, s>>>(t.cnt, h->tco, T + 1);
             if (h->dtype == DTC_FP16)
-                k_place<uint16_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
-                    M, csr->rowptr, h->rwo, t.rank, (const uint4*)t.mask, h->tco,
-                    (const uint16_t*)csr->vals, h->lid, (uint16_t*)h->vals);
+                k_fill_window<uint16_t><<<(unsigned)W, kFillThreads, 0, s>>>(
+                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, t.mask, (const uint16_t*)csr->vals,
+                    h->tco, h->lid, (uint16_t*)h->vals, h->atob);
             else
-                k_place<uint32_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
-                    M, csr->rowptr, h->rwo, t.rank, (const uint4*)t.mask, h->tco,
-                    (const uint32_t*)csr->vals, h->lid, (uint32_t*)h->vals);
+                k_fill_window<uint32_t><<<(unsigned)W, kFillThreads, 0, s>>>(
+                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, t.mask, (const uint32_t*)csr->vals,
+                    h->tco, h->lid, (uint32_t*)h->vals, h->atob);
         } else {
             TRYC(cudaMemsetAsync(h->tco, 0, sizeof(int32_t), s));
         }
         TRYC(cudaGetLastError());
+        st.mark("F3 fill");
         // F4: work units
         int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T, W);
         h->unit_blocks = U;
@@ -534,8 +566,10 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             k_units_fix<<<grid_for(h->num_units, 256, 4096), 256, 0, s>>>(h->num_units, W, h->rwo, h->units);
         }
         TRYC(cudaGetLastError());
+        st.mark("F4 units");
         t.release(s);
         TRYC(cudaStreamSynchronize(s));
+        st.mark("release temps");
         *out = h;
         return DTC_OK;
     }

@@ -72,16 +72,19 @@ void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* tmp
 
 inline int elt_size(int32_t dtype) { return dtype == DTC_FP16 ? 2 : 4; }
 
-// stream-ordered device allocation helpers (cudaMallocAsync pool)
+// Stream-ordered device allocations come from a library-owned memory pool per
+// device whose release threshold is "never": freed blocks stay cached, so a
+// second build / a growing workspace does not pay the OS map/unmap cost again.
+cudaMemPool_t lib_pool();
+
 template <class T>
 int dalloc(T** p, size_t count, cudaStream_t s) {
     *p = nullptr;
     if (count == 0) count = 1;
-    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(p), count * sizeof(T), s);
+    cudaError_t e = cudaMallocFromPoolAsync(reinterpret_cast<void**>(p), count * sizeof(T), lib_pool(), s);
     if (e != cudaSuccess) {
         cudaGetLastError();
-        set_error("device allocation of %zu bytes failed: %s", count * sizeof(T),
-                  cudaGetErrorString(e));
+        set_error("device allocation of %zu bytes failed: %s", count * sizeof(T), cudaGetErrorString(e));
         return DTC_ERR_OOM;
     }
     return DTC_OK;
@@ -91,6 +94,9 @@ void dfree(T*& p, cudaStream_t s) {
     if (p) cudaFreeAsync(reinterpret_cast<void*>(p), s);
     p = nullptr;
 }
+
+// small pinned host buffer (per thread) for the build's blocking scalar readbacks
+int64_t* pinned_scratch();
 
 int num_sms();
 

@@ -927,13 +927,21 @@ extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int6
     if (bbytes > h->stage_B_bytes) {
         dfree(h->stage_B, s);
         h->stage_B_bytes = 0;
-        DTC_CUDA(cudaMallocAsync(&h->stage_B, bbytes, s));
+        {
+            uint8_t* sb = nullptr;
+            int rc0 = dalloc(&sb, bbytes, s);
+            if (rc0) return rc0;
+            h->stage_B = sb;
+        }
         h->stage_B_bytes = bbytes;
     }
     if (cbytes > h->stage_C_bytes) {
         dfree(h->stage_C, s);
         h->stage_C_bytes = 0;
-        DTC_CUDA(cudaMallocAsync((void**)&h->stage_C, cbytes, s));
+        {
+            int rc0 = dalloc(&h->stage_C, cbytes / sizeof(float), s);
+            if (rc0) return rc0;
+        }
         h->stage_C_bytes = cbytes;
     }
     if (h->K > 0)

@@ -22,6 +22,37 @@ int cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
     return e == cudaErrorMemoryAllocation ? DTC_ERR_OOM : DTC_ERR_CUDA;
 }
 
+cudaMemPool_t lib_pool() {
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (!pools[dev]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            cudaGetLastError();
+            cudaDeviceGetDefaultMemPool(&p, dev);
+        }
+        uint64_t keep = ~uint64_t(0);
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &keep);
+        pools[dev] = p;
+    }
+    return pools[dev];
+}
+
+int64_t* pinned_scratch() {
+    static thread_local int64_t* buf = nullptr;
+    if (!buf && cudaMallocHost(reinterpret_cast<void**>(&buf), 64 * sizeof(int64_t)) != cudaSuccess) {
+        cudaGetLastError();
+        buf = nullptr;
+    }
+    return buf;
+}
+
 int num_sms() {
     int dev = 0, n = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) return 148;
