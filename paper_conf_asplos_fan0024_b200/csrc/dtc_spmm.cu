@@ -52,12 +52,28 @@ constexpr int ldg_prefetch() {
     return 1;
 #endif
 }
-template <int DT, int W>
+// per-thread register cap (sets occupancy) for a CTA of W consumer warps, each owning CW column
+// chunks -- from the measured sweeps (profiles/r01_design_evidence.md)
+template <int DT, int W, int CW>
 constexpr int ldg_maxregs() {
 #ifdef DTC_LDG_MAXREGS
-    return DTC_LDG_MAXREGS;
+    return DTC_LDG_MAXREGS * CW;
 #else
-    return 64;
+    return CW == 1 ? 64 : (W <= 2 ? 96 : 80);
+#endif
+}
+template <int DT, int W, int CW>
+constexpr int ldg_min_blocks() {
+    constexpr int b = 65536 / (W * 32 * ldg_maxregs<DT, W, CW>());
+    return b > 32 ? 32 : (b < 1 ? 1 : b);
+}
+// column chunks (of 32 fp32 / 64 fp16 columns) per consumer warp in the register-gather kernel
+template <int DT>
+constexpr int ldg_colchunks() {
+#ifdef DTC_TF32_CW
+    return DT == DTC_TF32 ? DTC_TF32_CW : 1;
+#else
+    return DT == DTC_TF32 ? 2 : 1;   // TF32 warps own 64 columns: one A-fragment read per 64 columns
 #endif
 }
 template <int DT, int W>
@@ -157,8 +173,13 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 
 // --------------------------------------------------- C tile store / split partials
 // A consumer warp owns rows (w*16 + g, w*16 + g + 8) and, for hi in {0,1} and
-// q < NJ/4, the 4 consecutive columns base + hi*HOFF + 4q (acc[4q..4q+3][2*half+hi]).
-template <int NJ, bool VEC>
+// quad q < NJ/4, the 4 consecutive columns base + hi*HOFF + col_of_quad(q)
+// (acc[4q..4q+3][2*half+hi]).  A warp may own CW column chunks of QPC quads each,
+// CSTRIDE columns apart: col_of_quad(q) = 4*(q % QPC) + CSTRIDE*(q / QPC).
+template <int QPC, int CSTRIDE>
+__device__ __forceinline__ int col_of_quad(int q) { return 4 * (q % QPC) + CSTRIDE * (q / QPC); }
+
+template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
 __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int64_t w, int g,
                                            int64_t base, int hoff, const float (&acc)[NJ][4], bool zero) {
 #pragma unroll
@@ -170,7 +191,7 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
         for (int hi = 0; hi < 2; ++hi) {
 #pragma unroll
             for (int q = 0; q < NJ / 4; ++q) {
-                const int64_t c = base + hi * hoff + 4 * q;
+                const int64_t c = base + hi * hoff + col_of_quad<QPC, CSTRIDE>(q);
                 float4 v;
                 v.x = zero ? 0.f : acc[4 * q + 0][2 * half + hi];
                 v.y = zero ? 0.f : acc[4 * q + 1][2 * half + hi];
@@ -190,7 +211,7 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
 }
 
 // Split-window fixup for one warp's tile (deterministic: slots summed in piece order).
-template <int NJ, bool VEC>
+template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
 __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
                                             int32_t* __restrict__ ctr, float* __restrict__ C, int64_t ldc, int64_t M,
                                             int64_t N, int g, int lane, int64_t base, int hoff) {
@@ -202,7 +223,7 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
         for (int hi = 0; hi < 2; ++hi)
 #pragma unroll
             for (int q = 0; q < NJ / 4; ++q) {
-                const int64_t c = base + hi * hoff + 4 * q;
+                const int64_t c = base + hi * hoff + col_of_quad<QPC, CSTRIDE>(q);
                 __stcg(reinterpret_cast<float4*>(prow + c),
                        make_float4(acc[4 * q + 0][2 * half + hi], acc[4 * q + 1][2 * half + hi],
                                    acc[4 * q + 2][2 * half + hi], acc[4 * q + 3][2 * half + hi]));
@@ -230,7 +251,7 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
             for (int hi = 0; hi < 2; ++hi)
 #pragma unroll
                 for (int q = 0; q < NJ / 4; ++q) {
-                    const int64_t c = base + hi * hoff + 4 * q;
+                    const int64_t c = base + hi * hoff + col_of_quad<QPC, CSTRIDE>(q);
                     const float4 v = __ldcg(reinterpret_cast<const float4*>(prow + c));
                     acc[4 * q + 0][2 * half + hi] += v.x;
                     acc[4 * q + 1][2 * half + hi] += v.y;
@@ -239,7 +260,7 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
                 }
         }
     }
-    store_tile<NJ, VEC>(C, ldc, M, N, u.wb, g, base, hoff, acc, false);
+    store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, u.wb, g, base, hoff, acc, false);
 }
 
 // --------------------------------------------------- S1: A batch producer (one warp)
@@ -512,14 +533,24 @@ __device__ __forceinline__ V16 load_b(const void* __restrict__ B, int64_t ldb, i
 // (the paper's sparse double buffering, made two-deep).  Each warp
 // streams its 32/64-column B slice with a kPrefetch-deep register ring that runs
 // continuously across chunk boundaries (VFetchDense + remap).
-template <int DT, int WARPS, bool VEC>
-__global__ void __launch_bounds__(WARPS * 32, (65536 / (WARPS * 32 * ldg_maxregs<DT, WARPS>())) > 32 ? 32 : (65536 / (WARPS * 32 * ldg_maxregs<DT, WARPS>())))
+// shared-memory bytes of the register-gather kernel (A chunks double buffered)
+template <int DT, int W>
+constexpr int ldg_smem_bytes() {
+    constexpr int S = ldg_chunk<DT, W>();
+    return 2 * S * 32 * Traits<DT>::FRAG_WORDS * 4 + 2 * S * 8 * 4 + 2 * (S + 1) * 4;
+}
+
+template <int DT, int WARPS, bool VEC, int CW>
+__global__ void __launch_bounds__(WARPS * 32, ldg_min_blocks<DT, WARPS, CW>())
 k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
            const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob, const void* __restrict__ avals,
            const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
     using Tr = Traits<DT>;
-    constexpr int NJ = Tr::NJ, COLW = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
+    constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
+    constexpr int NJ = NJ1 * CW;          // n8 mmas per TC block per warp (CW column chunks)
+    constexpr int COLW = COLW1 * CW;      // columns per warp
+    constexpr int QPC = NJ1 / 4;          // accumulator quads per column chunk
     constexpr int P = ldg_prefetch<DT, WARPS>();
     constexpr int S = ldg_chunk<DT, WARPS>();
     constexpr int NT = WARPS * 32;
@@ -537,8 +568,8 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     const int64_t n0 = ((int64_t)blockIdx.y * WARPS + warp) * COLW;
     const bool active = n0 < N;
     const int64_t bcol = n0 + (int64_t)VW * g;
-    const int64_t base = n0 + 2 * NJ * t;
-    const int hoff = NJ;
+    const int64_t base = n0 + 2 * NJ1 * t;
+    const int hoff = NJ1;
     const bool split = u.split_id >= 0;
     const int nblocks = u.be - u.bb;
     const int nchunks = (nblocks + S - 1) / S;
@@ -632,7 +663,7 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     int next_end = INT_MAX;
     if (!split) {
         while (cur < u.we && rwo[cur + 1] <= u.bb) {
-            if (active) store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+            if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true);
             ++cur;
         }
         next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
@@ -650,7 +681,8 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         if (nchunks > 1) ent_load_n(1, chunk_nb(1));
         if (nchunks > 2) meta_load(2);
 
-        V16 b0[P], b1[P];
+        {
+        V16 b0[P][CW], b1[P][CW];
         // thread's two B rows of block i: TF32 (t, t+4), FP16 (2t, 2t+1) -> adjacent id slots 2t, 2t+1
         auto ids_of = [&](int i) -> int2 {
             return *reinterpret_cast<const int2*>(s_ids + ((i / S) & 1) * S * 8 + (i % S) * 8 + 2 * t);
@@ -659,25 +691,28 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         // columns >= N are redirected to the zero line (no predication, no divergence)
         const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)sizeof(typename Tr::elt);
         const uint64_t ldb_bytes = (uint64_t)ldb * sizeof(typename Tr::elt);
-        const bool col_ok = bcol < N;
-        auto gather = [&](int row) -> V16 {
+        auto gather = [&](int row, int cw) -> V16 {
             if (VEC) {
-                const char* p = (row >= 0 && col_ok) ? bthr + (uint64_t)(uint32_t)row * ldb_bytes
-                                                     : reinterpret_cast<const char*>(g_zero_line);
+                const bool ok = row >= 0 && (bcol + cw * COLW1) < N;
+                const char* p = ok ? bthr + (uint64_t)(uint32_t)row * ldb_bytes + cw * COLW1 * (int)sizeof(typename Tr::elt)
+                                   : reinterpret_cast<const char*>(g_zero_line);
                 const uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
                 V16 v;
                 v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
                 return v;
             }
-            return load_b<DT, VEC>(B, ldb, row, bcol, N);
+            return load_b<DT, VEC>(B, ldb, row, bcol + cw * COLW1, N);
         };
         if (active) {
 #pragma unroll
             for (int q = 0; q < P; ++q) {
                 if (q < nblocks) {
                     const int2 id = ids_of(q);
-                    b0[q] = gather(id.x);
-                    b1[q] = gather(id.y);
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw) {
+                        b0[q][cw] = gather(id.x, cw);
+                        b1[q][cw] = gather(id.y, cw);
+                    }
                 }
             }
         }
@@ -693,30 +728,37 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
                             const uint4 av = reinterpret_cast<const uint4*>(fr)[lane];
                             const uint32_t a[4] = {av.x, av.y, av.z, av.w};
 #pragma unroll
-                            for (int jj = 0; jj < NJ; ++jj)
-                                mma_tf32(acc[jj], a, b0[q].w[jj], b1[q].w[jj]);
+                            for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                                for (int jj = 0; jj < NJ1; ++jj)
+                                    mma_tf32(acc[cw * NJ1 + jj], a, b0[q][cw].w[jj], b1[q][cw].w[jj]);
                         } else {
                             const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
                             const uint32_t a[2] = {av.x, av.y};
 #pragma unroll
-                            for (int jj = 0; jj < NJ; ++jj) {
-                                const uint32_t bb = __byte_perm(b0[q].w[jj >> 1], b1[q].w[jj >> 1],
-                                                                (jj & 1) ? 0x7632 : 0x5410);
-                                mma_f16(acc[jj], a, bb);
-                            }
+                            for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                                for (int jj = 0; jj < NJ1; ++jj) {
+                                    const uint32_t bb = __byte_perm(b0[q][cw].w[jj >> 1], b1[q][cw].w[jj >> 1],
+                                                                    (jj & 1) ? 0x7632 : 0x5410);
+                                    mma_f16(acc[cw * NJ1 + jj], a, bb);
+                                }
                         }
                         if (i + P < nblocks) {
                             const int2 id = ids_of(i + P);
-                            b0[q] = gather(id.x);
-                            b1[q] = gather(id.y);
+#pragma unroll
+                            for (int cw = 0; cw < CW; ++cw) {
+                                b0[q][cw] = gather(id.x, cw);
+                                b1[q][cw] = gather(id.y, cw);
+                            }
                         }
                         if (u.bb + i + 1 == next_end) {
-                            store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false);
+                            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false);
 #pragma unroll
                             for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
                             ++cur;
                             while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
-                                store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+                                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true);
                                 ++cur;
                             }
                             next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
@@ -736,14 +778,15 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
                 if (c + 3 < nchunks) meta_load(c + 3);
             }
         }
+        }
     }
     if (!active) return;
     if (!split) {
-        while (cur < u.we) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
         return;
     }
     int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
 }
 
 // ============================================================ host side
@@ -814,12 +857,16 @@ static cudaError_t launch_tma(const LaunchArgs& a, const CUtensorMap& map) {
     return cudaGetLastError();
 }
 
-template <int DT, int WARPS, bool VEC>
+template <int DT, int WARPS, bool VEC, int CW>
 static cudaError_t launch_ldg(const LaunchArgs& a) {
-    constexpr int S = ldg_chunk<DT, WARPS>();
-    const size_t smem = (size_t)2 * S * 32 * Traits<DT>::FRAG_WORDS * 4 + (size_t)2 * S * 8 * 4 + (size_t)2 * (S + 1) * 4;
+    const size_t smem = ldg_smem_bytes<DT, WARPS>();
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_spmm_ldg<DT, WARPS, VEC, CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr = true;
+    }
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
-    k_spmm_ldg<DT, WARPS, VEC><<<grid, WARPS * 32, smem, a.s>>>(a.h->units, a.h->rwo, a.h->tco, a.h->lid, a.h->atob,
+    k_spmm_ldg<DT, WARPS, VEC, CW><<<grid, WARPS * 32, smem, a.s>>>(a.h->units, a.h->rwo, a.h->tco, a.h->lid, a.h->atob,
                                                                 a.h->vals, a.B, a.ldb, a.C, a.ldc, a.h->M, a.N,
                                                                 a.h->ws, a.h->counters, a.npad);
     return cudaGetLastError();
@@ -835,11 +882,12 @@ static cudaError_t dispatch(int warps, bool tma, const LaunchArgs& a, const CUte
             default: return launch_tma<DT, 8, VEC>(a, map);
         }
     }
+    constexpr int CW = ldg_colchunks<DT>();
     switch (warps) {
-        case 1: return launch_ldg<DT, 1, VEC>(a);
-        case 2: return launch_ldg<DT, 2, VEC>(a);
-        case 4: return launch_ldg<DT, 4, VEC>(a);
-        default: return launch_ldg<DT, 8, VEC>(a);
+        case 1: return launch_ldg<DT, 1, VEC, CW>(a);
+        case 2: return launch_ldg<DT, 2, VEC, CW>(a);
+        case 4: return launch_ldg<DT, 4, VEC, CW>(a);
+        default: return launch_ldg<DT, 8, VEC, CW>(a);
     }
 }
 
@@ -860,7 +908,17 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     }
     const int elt = elt_size(h->dtype);
     const int VW = 16 / elt;
-    const int colw = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
+    // TMA needs a 16-byte aligned base and row pitch; a ragged N is fine (OOB columns zero-fill)
+    CUtensorMap map;
+    memset(&map, 0, sizeof(map));
+    bool tma = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && h->K < (int64_t(1) << 31) &&
+               N < (int64_t(1) << 31) && g_force_path == 2;
+    if (tma) tma = make_bmap(&map, B, h->K, N, ldb, h->dtype);
+    // columns per warp: the TMA path uses one 128-byte slice per warp, the register path CW slices
+    const int colw_tma = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
+    const int colw_ldg = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW * ldg_colchunks<DTC_FP16>()
+                                               : Traits<DTC_TF32>::COLW * ldg_colchunks<DTC_TF32>();
+    const int colw = tma ? colw_tma : colw_ldg;
     const int64_t need = (N + colw - 1) / colw;
     const int warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
     const int64_t gy64 = (N + (int64_t)warps * colw - 1) / ((int64_t)warps * colw);
@@ -886,12 +944,6 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
             h->ws_bytes = wsb;
         }
     }
-    // TMA needs a 16-byte aligned base and row pitch; a ragged N is fine (OOB columns zero-fill)
-    CUtensorMap map;
-    memset(&map, 0, sizeof(map));
-    bool tma = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && h->K < (int64_t(1) << 31) &&
-               N < (int64_t(1) << 31) && g_force_path != 1;
-    if (tma) tma = make_bmap(&map, B, h->K, N, ldb, h->dtype);
     // float4 C stores need an aligned C; the LDG path additionally needs B vectors
     const bool cvec = ((uintptr_t)C % 16 == 0) && (ldc % 4 == 0) && (N % 4 == 0);
     const bool bvec = ((uintptr_t)B % 16 == 0) && (ldb % VW == 0) && (N % VW == 0);
