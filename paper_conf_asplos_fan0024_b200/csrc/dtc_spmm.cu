@@ -59,7 +59,7 @@ constexpr int ldg_maxregs() {
 #ifdef DTC_LDG_MAXREGS
     return DTC_LDG_MAXREGS * CW;
 #else
-    return CW == 1 ? 64 : (W <= 2 ? 96 : 80);
+    return CW == 1 ? 64 : (DT == DTC_FP16 ? 112 : (W <= 2 ? 96 : 80));
 #endif
 }
 template <int DT, int W, int CW>
@@ -70,10 +70,16 @@ constexpr int ldg_min_blocks() {
 // column chunks (of 32 fp32 / 64 fp16 columns) per consumer warp in the register-gather kernel
 template <int DT>
 constexpr int ldg_colchunks() {
-#ifdef DTC_TF32_CW
-    return DT == DTC_TF32 ? DTC_TF32_CW : 1;
+#if defined(DTC_TF32_CW) || defined(DTC_FP16_CW)
+#ifndef DTC_TF32_CW
+#define DTC_TF32_CW 2
+#endif
+#ifndef DTC_FP16_CW
+#define DTC_FP16_CW 1
+#endif
+    return DT == DTC_TF32 ? DTC_TF32_CW : DTC_FP16_CW;
 #else
-    return DT == DTC_TF32 ? 2 : 1;   // TF32 warps own 64 columns: one A-fragment read per 64 columns
+    return 2;   // a warp owns 2 x 128-byte column slices: one A-fragment read per 64 fp32 / 128 fp16 columns
 #endif
 }
 template <int DT, int W>
