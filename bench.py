@@ -45,6 +45,7 @@ def parse_args():
     p.add_argument("--config", default="c2")
     p.add_argument("--n", type=int, default=0, help="override N (columns of B)")
     p.add_argument("--unit-blocks", type=int, default=0)
+    p.add_argument("--guided", type=int, default=0, help="F4 guided tail (1 on, 0 off)")
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
@@ -218,7 +219,8 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
         for _ in range(2):
             torch.cuda.synchronize()
             tb0 = time.perf_counter()
-            fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks)
+            fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks,
+                                   guided=args.guided)
             torch.cuda.synchronize()
             build_ms_runs.append((time.perf_counter() - tb0) * 1e3)
         build_ms = build_ms_runs[-1]

@@ -40,8 +40,9 @@ typedef enum {
 } dtc_status_t;
 
 /* Value / operand precision.
- * DTC_TF32: A values and B are fp32 in memory; the tensor cores multiply them
- *           rounded to TF32 (cvt.rna) with fp32 accumulation.
+ * DTC_TF32: A values and B are fp32 in memory; A is rounded to TF32 (cvt.rna)
+ *           when staged, B is fed to the tensor core as fp32 bits (TF32 truncation);
+ *           fp32 accumulation (error budget in DESIGN.md C13).
  * DTC_FP16: A values and B are fp16 in memory; fp32 accumulation; C is fp32.   */
 typedef enum { DTC_TF32 = 0, DTC_FP16 = 1 } dtc_dtype_t;
 
@@ -66,7 +67,8 @@ typedef struct dtc_format* dtc_handle_t;   /* opaque, library-owned */
  *   tc_local_id       uint8[nnz]            row_in_window*8 + col_in_block (<128)
  *   sparse_a_to_b     int32[8T]             original column of each block column, -1 pad
  *   tc_values         dtype[nnz]            values aligned with tc_local_id
- *   units             int32[8*num_units]    F4 work-unit table (see dtc_schedule_export) */
+ *   units             int32[8*num_units]    F4 work units {wb, we, bb, be, split_id, piece,
+ *                                            npieces, slot_base} (see dtc_format_export) */
 typedef struct {
     int64_t M, K, nnz, num_windows, num_tc_blocks, num_units, num_split_windows;
     int32_t dtype;
@@ -80,12 +82,15 @@ typedef struct {
 } dtc_format_view_t;
 
 /* Build options (zero-initialised = defaults).
- *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T and the SM count
+ *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T, W and the SM count
  *   dedup_path   F1 per-window dedup: 0 auto, 1 force smem sort, 2 force chunked bitmap
- *                (both produce bit-identical formats; exposed for tests) */
+ *                (both produce bit-identical formats; exposed for tests)
+ *   guided       F4 tail: 0 = fixed-size units (default); 1 = units of U/2 over the last
+ *                ~half wave of TC blocks (measured: +-1% on large matrices, -8% on c2) */
 typedef struct {
     int32_t unit_blocks;
     int32_t dedup_path;
+    int32_t guided;
 } dtc_build_opts_t;
 
 /* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on

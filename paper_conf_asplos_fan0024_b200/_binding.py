@@ -40,7 +40,7 @@ class _View(ctypes.Structure):
 
 
 class _Opts(ctypes.Structure):
-    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32)]
+    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32)]
 
 
 class DtcError(RuntimeError):
@@ -166,10 +166,10 @@ class Format:
 
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
-              unit_blocks: int = 0, dedup_path: int = 0) -> "Format":
+              unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0) -> "Format":
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
         h = ctypes.c_void_p()
-        opts = _Opts(int(unit_blocks), int(dedup_path))
+        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value)

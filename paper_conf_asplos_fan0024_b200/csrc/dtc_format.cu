@@ -310,22 +310,60 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
 
 // ---------------------------------------------------------------- F4
 // Work units: consecutive windows whose first TC block falls in
-// the same U-block chunk form one unit; a window with more than U blocks is
-// split into ceil(nb/U) near-equal pieces (each its own unit, deterministic fixup).
-__global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, int U,
+// the same chunk form one unit; a window with more blocks than its chunk size is
+// split into near-equal pieces (each its own unit, deterministic fixup).  Chunk
+// sizes are "guided": U blocks, then U/2, U/4, U/8 over the last ~one wave of
+// blocks, so the CTAs dispatched last are short and the tail of the grid is even.
+struct Guide {
+    int64_t x[5];     // segment starts (x[4] = T)
+    int64_t sz[4];    // chunk size per segment
+    int64_t off[4];   // chunk-id offset per segment
+    __host__ __device__ int seg(int64_t v) const {
+        int k = 0;
+        while (k < 3 && v >= x[k + 1]) ++k;
+        return k;
+    }
+    __host__ __device__ int64_t chunk(int64_t v) const {
+        const int k = seg(v);
+        return off[k] + (v - x[k]) / sz[k];
+    }
+    __host__ __device__ int64_t size_at(int64_t v) const { return sz[seg(v)]; }
+};
+
+static Guide make_guide(int64_t T, int U, int64_t tail_span) {
+    Guide g;
+    int64_t A = tail_span > T ? T : tail_span;
+    g.x[0] = 0;
+    g.x[1] = T - A;
+    g.x[2] = T - A / 2;
+    g.x[3] = T - A / 4;
+    g.x[4] = T;
+    // sizes U, then U/2 for the rest of the tail (smaller units lose more to per-unit
+    // startup than they win at the end of the grid -- measured)
+    for (int k = 0; k < 4; ++k) {
+        const int64_t sz = k == 0 ? U : U / 2;
+        g.sz[k] = sz < 8 ? 8 : sz;
+    }
+    g.off[0] = 0;
+    for (int k = 1; k < 4; ++k) g.off[k] = g.off[k - 1] + (g.x[k] - g.x[k - 1] + g.sz[k - 1] - 1) / g.sz[k - 1];
+    return g;
+}
+
+__global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, Guide gd,
                               int64_t* __restrict__ cnt, int64_t* __restrict__ split,
                               int64_t* __restrict__ slots) {
     for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
-        int64_t nb = rwo[w + 1] - rwo[w];
-        bool big = nb > U;
+        const int64_t nb = rwo[w + 1] - rwo[w];
+        const int64_t U = gd.size_at(rwo[w]);
+        const bool big = nb > U;
         int64_t c;
         if (big) {
             c = (nb + U - 1) / U;
         } else {
             bool starts = (w == 0);
             if (!starts) {
-                int64_t pnb = rwo[w] - rwo[w - 1];
-                starts = (pnb > U) || (rwo[w] / U != rwo[w - 1] / U);
+                const int64_t pnb = rwo[w] - rwo[w - 1];
+                starts = (pnb > gd.size_at(rwo[w - 1])) || (gd.chunk(rwo[w]) != gd.chunk(rwo[w - 1]));
             }
             c = starts ? 1 : 0;
         }
@@ -335,14 +373,14 @@ __global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, int U,
     }
 }
 
-__global__ void k_units_fill(int64_t W, const int32_t* __restrict__ rwo, int U,
+__global__ void k_units_fill(int64_t W, const int32_t* __restrict__ rwo, Guide gd,
                              const int64_t* __restrict__ ubase, const int64_t* __restrict__ sbase,
                              const int64_t* __restrict__ slbase, Unit* __restrict__ units) {
     for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < W; w += (int64_t)gridDim.x * blockDim.x) {
         int64_t c = ubase[w + 1] - ubase[w];
         if (c == 0) continue;
         int64_t nb = rwo[w + 1] - rwo[w];
-        if (nb > U) {
+        if (nb > gd.size_at(rwo[w])) {
             for (int64_t p = 0; p < c; ++p) {
                 Unit u;
                 u.wb = (int32_t)w; u.we = (int32_t)(w + 1);
@@ -544,11 +582,14 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         // F4: work units
         int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T, W);
         h->unit_blocks = U;
+        // optional guided tail over about half a wave of units (opts->guided > 0)
+        const int64_t tail = (opts && opts->guided > 0) ? (int64_t)num_sms() * 4 * U : 0;
+        const Guide gd = make_guide(T, U, tail);
         if (W > 0) {
             TRY(dalloc(&t.ucnt, W + 1, s));
             TRY(dalloc(&t.usplit, W + 1, s));
             TRY(dalloc(&t.uslots, W + 1, s));
-            k_units_count<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, U, t.ucnt, t.usplit, t.uslots);
+            k_units_count<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, gd, t.ucnt, t.usplit, t.uslots);
             dfree(t.scan_tmp, s);
             TRY(dalloc(&t.scan_tmp, scan_tmp_elems(W + 1) + 64, s));
             exclusive_scan_i64(t.ucnt, t.ucnt, W, t.scan_tmp, s);
@@ -562,7 +603,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             h->num_split = t.host[3];
             h->num_slots = t.host[4];
             TRY(dalloc(&h->units, std::max<int64_t>(h->num_units, 1), s));
-            k_units_fill<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, U, t.ucnt, t.usplit, t.uslots, h->units);
+            k_units_fill<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, gd, t.ucnt, t.usplit, t.uslots, h->units);
             k_units_fix<<<grid_for(h->num_units, 256, 4096), 256, 0, s>>>(h->num_units, W, h->rwo, h->units);
         }
         TRYC(cudaGetLastError());
