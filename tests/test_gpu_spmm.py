@@ -213,3 +213,25 @@ def test_config_full_size(name, N):
     # all columns of a few whole rows, including the last (tail window) row
     for r0 in (0, cfg.M - 3):
         check_tol(C[r0:r0 + 3], cfg.M, cfg.K, rp, ci, v, B, cfg.dtype, r0=r0, r1=r0 + 3)
+
+
+@pytest.mark.parametrize("name,N", [("c3", 256), ("c3h", 256), ("c4", 128), ("c5", 512)])
+def test_p2_integer_full_size_sampled_exact(name, N):
+    """P2 at full size: integer A and B (|a|,|b| <= 4 -> every product and partial sum is
+    exact in TF32/FP16 and FP32 as long as row sums stay below 2^24; the largest rows here
+    give < 2^20), so sampled GPU entries must EQUAL the FP64 oracle, in the bench's launch
+    configuration (default unit size, vector path)."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.integers(cfg.seed_a, 5, len(ci), -2, 2)
+    B = datagen.integers(cfg.seed_b, 6, cfg.K * N, -2, 2).reshape(cfg.K, N)
+    if cfg.dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=cfg.dtype)
+    C = spmm(f, B)
+    rng = np.random.default_rng(1)
+    rows = _sample(cfg, rp, rng, n=8192)
+    cols = rng.integers(0, N, size=len(rows)).astype(np.int64)
+    Cr, Bd = oracle.spmm_at(cfg.M, rp, ci, v.astype(np.float32), B.astype(np.float32), rows, cols)
+    assert float(Bd.max()) < 2 ** 23
+    assert np.array_equal(C[rows, cols].astype(np.float64), Cr)
