@@ -324,6 +324,37 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
         # parity spot check of the timed result (sampled, oracle lives in tests; here a cheap self-check)
         out["e2e_matches_device"] = bool(torch.equal(Ch, C_d.cpu()))
 
+    # ---- e2e at N > 1: root copies B from pinned host memory, dtc_spmm_dist broadcasts it over
+    # NCCL and runs the local row windows, every rank reads its C rows back; max over ranks
+    if not args.no_e2e and world > 1:
+        import torch.distributed as tdist
+        Bh = torch.from_numpy(B).pin_memory() if rank == 0 else None
+        Ch = torch.empty(tuple(C_d.shape), dtype=torch.float32).pin_memory()
+
+        def e2e_step():
+            if rank == 0:
+                B_d.copy_(Bh, non_blocking=True)
+            dd.spmm(B_d, C_d, root=0, gather_c=False)
+            Ch.copy_(C_d, non_blocking=True)
+            torch.cuda.synchronize()
+
+        for _ in range(2):
+            e2e_step()
+        tdist.barrier()
+        e2e_steps = max(3, min(args.steps, 20))
+        t0 = time.perf_counter()
+        for _ in range(e2e_steps):
+            e2e_step()
+        el = torch.tensor([(time.perf_counter() - t0) / e2e_steps], device=dev)
+        tdist.all_reduce(el, op=tdist.ReduceOp.MAX)
+        e2e_s = float(el.item())
+        out["e2e"] = {"value": round(flops / e2e_s / 1e9, 2), "unit": UNIT,
+                      "h2d_bytes_per_step": int(B.nbytes), "d2h_bytes_per_step": int(M * N * 4),
+                      "ms_per_step": round(e2e_s * 1e3, 4),
+                      "api": "dtc_spmm_dist (root H2D of B, NCCL broadcast, local kernel, per-rank C D2H)",
+                      "steps": e2e_steps}
+        out["format_build_ms"] = round(build_ms, 3)
+
     # ---- cuSPARSE on the same box (comparison system)
     if not args.no_cusparse and world == 1:
         try:
