@@ -177,6 +177,31 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
 }
 
+// L2 eviction-priority hints (experiment DTC_L2_HINTS): B gathers evict_last, streamed data
+// (C stores) evict_first, so reusable B rows survive the streaming traffic in L2.
+#ifdef DTC_L2_HINTS
+__device__ __forceinline__ uint64_t l2_policy_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint4 ldg_hint(const void* ptr, uint64_t pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(ptr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ void stg_hint(void* ptr, float4 v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1,%2,%3,%4}, %5;"
+                 :: "l"(ptr), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol) : "memory");
+}
+#endif
+
 // --------------------------------------------------- C tile store / split partials
 // A consumer warp owns rows (w*16 + g, w*16 + g + 8) and, for hi in {0,1} and
 // quad q < NJ/4, the 4 consecutive columns base + hi*HOFF + col_of_quad(q)
@@ -204,7 +229,11 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
                 v.z = zero ? 0.f : acc[4 * q + 2][2 * half + hi];
                 v.w = zero ? 0.f : acc[4 * q + 3][2 * half + hi];
                 if (VEC) {
+#if defined(DTC_L2_HINTS) && (DTC_L2_HINTS & 2)
+                    if (c < N) stg_hint(crow + c, v, l2_policy_first());
+#else
                     if (c < N) *reinterpret_cast<float4*>(crow + c) = v;
+#endif
                 } else {
                     if (c + 0 < N) crow[c + 0] = v.x;
                     if (c + 1 < N) crow[c + 1] = v.y;
@@ -697,12 +726,19 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         // columns >= N are redirected to the zero line (no predication, no divergence)
         const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)sizeof(typename Tr::elt);
         const uint64_t ldb_bytes = (uint64_t)ldb * sizeof(typename Tr::elt);
+#if defined(DTC_L2_HINTS) && (DTC_L2_HINTS & 1)
+        const uint64_t pol_b = l2_policy_last();
+#endif
         auto gather = [&](int row, int cw) -> V16 {
             if (VEC) {
                 const bool ok = row >= 0 && (bcol + cw * COLW1) < N;
                 const char* p = ok ? bthr + (uint64_t)(uint32_t)row * ldb_bytes + cw * COLW1 * (int)sizeof(typename Tr::elt)
                                    : reinterpret_cast<const char*>(g_zero_line);
+#if defined(DTC_L2_HINTS) && (DTC_L2_HINTS & 1)
+                const uint4 x = ldg_hint(p, pol_b);
+#else
                 const uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
+#endif
                 V16 v;
                 v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
                 return v;
@@ -910,7 +946,10 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     if (h->num_units == 0) return DTC_OK;
     if (g_force_path < 0) {
         const char* e = getenv("DTC_SPMM_PATH");
-        g_force_path = (e && e[0] == 't') ? 2 : 1;   // default: register gather (see header)
+#ifndef DTC_DEFAULT_PATH
+#define DTC_DEFAULT_PATH 1
+#endif
+        g_force_path = (e && e[0] == 't') ? 2 : (e && e[0] == 'l') ? 1 : DTC_DEFAULT_PATH;   // default: register gather
     }
     const int elt = elt_size(h->dtype);
     const int VW = 16 / elt;
