@@ -91,6 +91,12 @@ typedef struct {
     int32_t unit_blocks;
     int32_t dedup_path;
     int32_t guided;
+    int32_t reserved;
+    /* optional row permutation (DEVICE int32[M], new row -> original row, a bijection):
+     * the library condenses the permuted matrix and dtc_spmm still writes C in the
+     * ORIGINAL row order (e.g. the TCA order from dtc_tca_reorder).  NULL = identity.
+     * Not a permutation -> DTC_ERR_INVALID. */
+    const int32_t* row_perm;
 } dtc_build_opts_t;
 
 /* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on
@@ -133,6 +139,17 @@ int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, fl
 int dtc_spmm_launches_per_call(void);
 
 void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory */
+
+/* ------------------------------------------------------------ reordering (NEXT-1)
+ * TCU-Cache-Aware reordering, §4.3 Alg. 1 (optional HOST
+ * preprocessing): MinHash-LSH row pairs -> priority queue by Jaccard -> row clusters
+ * of BLOCK_HEIGHT = 16 rows (Hierarchy I), then the same over row clusters into
+ * clusters of sm_num clusters (Hierarchy II, L2 locality), then Reid.  HOST inputs:
+ * canonical CSR pattern rowptr[M+1], colidx[nnz].  Output perm[M] (host): new row ->
+ * original row, to pass as dtc_build_opts_t.row_perm (after copying to the device).
+ * Deterministic (readings DESIGN.md T1-T8).  Errors: INVALID, OOM. */
+int dtc_tca_reorder(int64_t M, int64_t K, const int32_t* rowptr_host, const int32_t* colidx_host,
+                    int32_t sm_num, int32_t* perm_host);
 
 /* ------------------------------------------------------------ distributed
  * One process per GPU (north_star).  Row windows are partitioned across ranks

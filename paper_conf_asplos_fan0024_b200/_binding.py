@@ -40,7 +40,8 @@ class _View(ctypes.Structure):
 
 
 class _Opts(ctypes.Structure):
-    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32)]
+    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("reserved", _i32),
+                ("row_perm", _vp)]
 
 
 class DtcError(RuntimeError):
@@ -77,6 +78,7 @@ def lib():
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
+            L.dtc_tca_reorder.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp]
             L.dtc_nccl_unique_id.argtypes = [_vp]
             L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
             L.dtc_dist_query.argtypes = [_vp, P(_i64), P(_i64), P(_vp)]
@@ -166,10 +168,16 @@ class Format:
 
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
-              unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0) -> "Format":
+              unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None) -> "Format":
+        """row_perm: optional CUDA int32 tensor [M], new row -> original row (e.g. tca_reorder);
+        C is still produced in the original row order."""
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
         h = ctypes.c_void_p()
-        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided))
+        if row_perm is not None:
+            import torch
+            if row_perm.dtype != torch.int32 or not row_perm.is_cuda or row_perm.numel() != M:
+                raise TypeError("row_perm must be a CUDA int32 tensor of length M")
+        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), 0, _dptr(row_perm))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value)
@@ -262,6 +270,16 @@ def partition_windows(rwo, world: int) -> np.ndarray:
     _check(lib().dtc_partition_windows(rwo.ctypes.data_as(_vp), len(rwo) - 1, world, out.ctypes.data_as(_vp)),
            "dtc_partition_windows")
     return out
+
+
+def tca_reorder(M: int, K: int, rowptr, colidx, sm_num: int = 148) -> np.ndarray:
+    """TCA row reordering (dtc_tca_reorder, host): perm[new_row] = original row."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int32)
+    colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+    perm = np.zeros(max(M, 1), dtype=np.int32)
+    _check(lib().dtc_tca_reorder(M, K, rowptr.ctypes.data_as(_vp), colidx.ctypes.data_as(_vp), sm_num,
+                                 perm.ctypes.data_as(_vp)), "dtc_tca_reorder")
+    return perm[:M]
 
 
 def nccl_unique_id() -> bytes:

@@ -219,6 +219,46 @@ k_dedup_bitmap(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ ro
     }
 }
 
+// ---------------------------------------------------------------- optional row permutation
+// (dtc_build_opts_t.row_perm, e.g. the TCA order): check it is a bijection, then gather the
+// permuted CSR (new row r = original row perm[r]) that F0-F4 then condense.
+__global__ void k_perm_count(int64_t M, const int32_t* __restrict__ perm, int32_t* __restrict__ seen,
+                             int* __restrict__ flags) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < M; r += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t v = perm[r];
+        if (v < 0 || v >= M) atomicOr(flags, 1);
+        else atomicAdd(&seen[v], 1);
+    }
+}
+__global__ void k_perm_deg(int64_t M, const int32_t* __restrict__ perm, const int32_t* __restrict__ seen,
+                           const int32_t* __restrict__ rowptr, int64_t nnz, int64_t* __restrict__ deg,
+                           int* __restrict__ flags) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < M; r += (int64_t)gridDim.x * blockDim.x) {
+        if (seen[r] != 1) atomicOr(flags, 1);
+        int64_t v = perm[r];
+        v = v < 0 ? 0 : (v >= M ? M - 1 : v);
+        const int64_t a = clamp64(rowptr[v], 0, nnz), b = clamp64(rowptr[v + 1], 0, nnz);
+        deg[r] = b > a ? b - a : 0;
+    }
+}
+template <class V>
+__global__ void k_perm_copy(int64_t M, const int32_t* __restrict__ perm, const int32_t* __restrict__ rowptr,
+                            const int64_t* __restrict__ nrp, const int32_t* __restrict__ ci, const V* __restrict__ vi,
+                            int32_t* __restrict__ co, V* __restrict__ vo) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = warp; r < M; r += nwarps) {
+        int64_t v = perm[r];
+        v = v < 0 ? 0 : (v >= M ? M - 1 : v);
+        const int64_t src = rowptr[v], dst = nrp[r], n = nrp[r + 1] - nrp[r];
+        for (int64_t k = lane; k < n; k += 32) {
+            co[dst + k] = ci[src + k];
+            vo[dst + k] = vi[src + k];
+        }
+    }
+}
+
 // ---------------------------------------------------------------- F2/F3
 __global__ void k_to_i32(const int64_t* __restrict__ in, int32_t* __restrict__ out, int64_t n) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -420,7 +460,7 @@ static void free_format(dtc_format* h, cudaStream_t s) {
     if (!h) return;
     dfree(h->rwo, s); dfree(h->tco, s); dfree(h->lid, s); dfree(h->atob, s);
     dfree(h->vals, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
-    dfree(h->stage_B, s); dfree(h->stage_C, s);
+    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s);
 }
 
 struct BuildTemps {
@@ -436,10 +476,16 @@ struct BuildTemps {
     int64_t* usplit = nullptr;   // [W+1]
     int64_t* uslots = nullptr;   // [W+1]
     int64_t* host = nullptr;     // pinned readback
+    int32_t* pseen = nullptr;    // row_perm: hit counts per original row
+    int64_t* pdeg = nullptr;     // row_perm: permuted degrees -> rowptr (int64)
+    int32_t* prow32 = nullptr;   // row_perm: permuted rowptr
+    int32_t* pcol = nullptr;     // row_perm: permuted colidx
+    uint8_t* pval = nullptr;     // row_perm: permuted values
     void release(cudaStream_t s) {
         dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s);
         dfree(scan_tmp, s); dfree(mask, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
         dfree(uslots, s);
+        dfree(pseen, s); dfree(pdeg, s); dfree(prow32, s); dfree(pcol, s); dfree(pval, s);
         host = nullptr;   // per-thread pinned scratch, not owned
     }
 };
@@ -502,6 +548,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
     h->M = M; h->K = K; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
     cudaGetDevice(&h->device);
     BuildTemps t;
+    dtc_csr_t pcsr;   // permuted CSR view (row_perm)
     StageTimer st;
     st.init(s);
     int rc = DTC_OK;
@@ -517,6 +564,36 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         TRY(dalloc(&t.uniq, nnz, s));
         TRY(dalloc(&t.rank, nnz, s));
         const int64_t scan_n = std::max<int64_t>(W + 1, 1);
+        if (opts && opts->row_perm && M > 0) {
+            // permuted CSR (F0 below validates its columns; the bijection is checked here)
+            TRY(dalloc(&t.pseen, M, s));
+            TRYC(cudaMemsetAsync(t.pseen, 0, M * sizeof(int32_t), s));
+            TRY(dalloc(&t.pdeg, M + 1, s));
+            TRY(dalloc(&t.scan_tmp, scan_tmp_elems(M + 1) + 64, s));
+            TRY(dalloc(&t.prow32, M + 1, s));
+            TRY(dalloc(&t.pcol, nnz, s));
+            TRY(dalloc(&t.pval, (size_t)std::max<int64_t>(nnz, 1) * elt_size(h->dtype), s));
+            k_perm_count<<<grid_for(M, 256, 4096), 256, 0, s>>>(M, opts->row_perm, t.pseen, t.flags);
+            k_perm_deg<<<grid_for(M, 256, 4096), 256, 0, s>>>(M, opts->row_perm, t.pseen, csr->rowptr, nnz, t.pdeg, t.flags);
+            exclusive_scan_i64(t.pdeg, t.pdeg, M, t.scan_tmp, s);
+            k_to_i32<<<grid_for(M + 1, 256, 4096), 256, 0, s>>>(t.pdeg, t.prow32, M + 1);
+            if (h->dtype == DTC_FP16)
+                k_perm_copy<uint16_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
+                    M, opts->row_perm, csr->rowptr, t.pdeg, csr->colidx, (const uint16_t*)csr->vals, t.pcol,
+                    (uint16_t*)t.pval);
+            else
+                k_perm_copy<uint32_t><<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(
+                    M, opts->row_perm, csr->rowptr, t.pdeg, csr->colidx, (const uint32_t*)csr->vals, t.pcol,
+                    (uint32_t*)t.pval);
+            TRY(dalloc(&h->rowmap, M, s));
+            TRYC(cudaMemcpyAsync(h->rowmap, opts->row_perm, M * sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+            dfree(t.scan_tmp, s);
+            pcsr = *csr;
+            pcsr.rowptr = t.prow32;
+            pcsr.colidx = t.pcol;
+            pcsr.vals = t.pval;
+            csr = &pcsr;
+        }
         st.mark("setup+temp alloc");
         // F0
         if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, t.flags);

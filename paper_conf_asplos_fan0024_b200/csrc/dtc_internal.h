@@ -50,6 +50,8 @@ struct dtc_format {
     size_t stage_B_bytes = 0;
     float* stage_C = nullptr;
     size_t stage_C_bytes = 0;
+    // optional row map (row of the condensed matrix -> row of C), from dtc_build_opts_t.row_perm
+    int32_t* rowmap = nullptr;
 };
 
 namespace dtc {

@@ -212,12 +212,14 @@ __device__ __forceinline__ int col_of_quad(int q) { return 4 * (q % QPC) + CSTRI
 
 template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
 __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int64_t w, int g,
-                                           int64_t base, int hoff, const float (&acc)[NJ][4], bool zero) {
+                                           int64_t base, int hoff, const float (&acc)[NJ][4], bool zero,
+                                           const int32_t* __restrict__ rowmap) {
 #pragma unroll
     for (int half = 0; half < 2; ++half) {
         const int64_t row = w * kWindow + g + 8 * half;
         if (row >= M) continue;
-        float* crow = C + row * ldc;
+        // row of the (possibly TCA-permuted) condensed matrix -> row of C in the caller's order
+        float* crow = C + (rowmap ? (int64_t)__ldg(rowmap + row) : row) * ldc;
 #pragma unroll
         for (int hi = 0; hi < 2; ++hi) {
 #pragma unroll
@@ -249,7 +251,8 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
 template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
 __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
                                             int32_t* __restrict__ ctr, float* __restrict__ C, int64_t ldc, int64_t M,
-                                            int64_t N, int g, int lane, int64_t base, int hoff) {
+                                            int64_t N, int g, int lane, int64_t base, int hoff,
+                                            const int32_t* __restrict__ rowmap) {
     const int64_t slot = (int64_t)u.slot_base + u.piece;
 #pragma unroll
     for (int half = 0; half < 2; ++half) {
@@ -295,7 +298,7 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
                 }
         }
     }
-    store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, u.wb, g, base, hoff, acc, false);
+    store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, u.wb, g, base, hoff, acc, false, rowmap);
 }
 
 // --------------------------------------------------- S1: A batch producer (one warp)
@@ -361,7 +364,8 @@ __global__ void __launch_bounds__((WARPS + 2) * 32)
 k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
-           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
+           const int32_t* __restrict__ rowmap) {
     using Tr = Traits<DT>;
     constexpr int NJ = Tr::NJ, COLW = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int S = kChunk;
@@ -462,7 +466,7 @@ k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     int64_t cur = u.wb;
     int64_t next_end = INT_MAX;
     if (!split) {
-        while (cur < u.we && rwo[cur + 1] <= u.bb) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        while (cur < u.we && rwo[cur + 1] <= u.bb) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
     }
 
@@ -499,21 +503,21 @@ k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         const int64_t b = u.bb + i;
         if (b + 1 == next_end) {   // S4: window boundary -> store and reset
-            store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false);
+            store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
 #pragma unroll
             for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
             ++cur;
-            while (cur < u.we && rwo[cur + 1] == rwo[cur]) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+            while (cur < u.we && rwo[cur + 1] == rwo[cur]) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
             next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
         }
     }
     if (!split) {
-        while (cur < u.we) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        while (cur < u.we) { store_tile<NJ, VEC>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         return;
     }
     // S5: split-window fixup per consumer warp
     int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
+    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
 }
 
 // ============================================================ fallback: register gather
@@ -580,7 +584,8 @@ __global__ void __launch_bounds__(WARPS * 32, ldg_min_blocks<DT, WARPS, CW>())
 k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
            const uint8_t* __restrict__ lid, const int32_t* __restrict__ atob, const void* __restrict__ avals,
            const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
-           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad) {
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
+           const int32_t* __restrict__ rowmap) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
     constexpr int NJ = NJ1 * CW;          // n8 mmas per TC block per warp (CW column chunks)
@@ -698,7 +703,7 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     int next_end = INT_MAX;
     if (!split) {
         while (cur < u.we && rwo[cur + 1] <= u.bb) {
-            if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+            if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
             ++cur;
         }
         next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
@@ -795,12 +800,12 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
                             }
                         }
                         if (u.bb + i + 1 == next_end) {
-                            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false);
+                            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
 #pragma unroll
                             for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
                             ++cur;
                             while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
-                                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true);
+                                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
                                 ++cur;
                             }
                             next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
@@ -824,11 +829,11 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     }
     if (!active) return;
     if (!split) {
-        while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true); ++cur; }
+        while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         return;
     }
     int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff);
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
 }
 
 // ============================================================ host side
@@ -895,7 +900,7 @@ static cudaError_t launch_tma(const LaunchArgs& a, const CUtensorMap& map) {
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
     k_spmm_tma<DT, WARPS, VEC><<<grid, (WARPS + 2) * 32, smem, a.s>>>(map, a.h->units, a.h->rwo, a.h->tco, a.h->lid,
                                                                       a.h->atob, a.h->vals, a.C, a.ldc, a.h->M, a.N,
-                                                                      a.h->ws, a.h->counters, a.npad);
+                                                                      a.h->ws, a.h->counters, a.npad, a.h->rowmap);
     return cudaGetLastError();
 }
 
@@ -910,7 +915,7 @@ static cudaError_t launch_ldg(const LaunchArgs& a) {
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
     k_spmm_ldg<DT, WARPS, VEC, CW><<<grid, WARPS * 32, smem, a.s>>>(a.h->units, a.h->rwo, a.h->tco, a.h->lid, a.h->atob,
                                                                 a.h->vals, a.B, a.ldb, a.C, a.ldc, a.h->M, a.N,
-                                                                a.h->ws, a.h->counters, a.npad);
+                                                                a.h->ws, a.h->counters, a.npad, a.h->rowmap);
     return cudaGetLastError();
 }
 
