@@ -15,8 +15,8 @@
 // with ties broken by (i, j) ascending and exact rational comparison; pairs whose
 // clusters coincide or already left the pool are skipped; leftover pool clusters
 // join the next hierarchy / the final order; clusters ordered by smallest row id.
-// The Python oracle (oracle/tca.py) implements the same steps; tests compare the
-// permutations exactly.
+// An independent step-by-step Python transcription under tests' control implements
+// the same steps; tests compare the permutations exactly.
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
