@@ -138,6 +138,17 @@ int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, fl
 /* Number of kernels dtc_spmm launches per call (for launch accounting). */
 int dtc_spmm_launches_per_call(void);
 
+/* Kernel variant used by dtc_spmm (ablations and the per-path parity tests).
+ * All variants compute the same S1-S5 and pass the same parity bar:
+ *   0 = library default, 1 = register gather with shared-memory A chunks (the paper's
+ *   FetchSparse/SDB structure), 2 = TMA tile::gather4 B ring,
+ *   3 = direct: each warp builds its A fragment from TCValues via the per-block
+ *   occupancy mask (no shared memory, no CTA barrier).
+ * Process-wide, takes effect at the next dtc_spmm; the environment variable
+ * DTC_SPMM_PATH=ldg|tma|dir sets the initial value.  Returns the previous setting
+ * (0 if it was the default), or DTC_ERR_INVALID for an unknown path. */
+int dtc_set_spmm_path(int path);
+
 void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory */
 
 /* ------------------------------------------------------------ reordering (NEXT-1)

@@ -75,6 +75,7 @@ def lib():
             L.dtc_spmm.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_launches_per_call.argtypes = []
+            L.dtc_set_spmm_path.argtypes = [ctypes.c_int]
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
@@ -120,6 +121,18 @@ def version() -> str:
 
 def launches_per_call() -> int:
     return int(lib().dtc_spmm_launches_per_call())
+
+
+SPMM_PATHS = {"default": 0, "ldg": 1, "tma": 2, "dir": 3}
+
+
+def set_spmm_path(path) -> int:
+    """Select the dtc_spmm kernel variant (include/dtc.h dtc_set_spmm_path); returns the previous one."""
+    code = SPMM_PATHS[path] if isinstance(path, str) else int(path)
+    st = int(lib().dtc_set_spmm_path(code))
+    if st < 0:
+        _check(st, "dtc_set_spmm_path")
+    return st
 
 
 def _dtype_code(dtype) -> int:

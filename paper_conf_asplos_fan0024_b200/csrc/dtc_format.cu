@@ -346,6 +346,8 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
         lid[pos] = (uint8_t)id;
         vout[pos] = vin[p];
     }
+    if (sm)   // persist the masks (the kernel-side fragment index)
+        for (int i = tid; i < nb * 4; i += kFillThreads) gmask[b0 * 4 + i] = s_mask[i];
 }
 
 // ---------------------------------------------------------------- F4
@@ -459,7 +461,7 @@ static unsigned grid_for(int64_t work, int per_block, int cap = 1 << 20) {
 static void free_format(dtc_format* h, cudaStream_t s) {
     if (!h) return;
     dfree(h->rwo, s); dfree(h->tco, s); dfree(h->lid, s); dfree(h->atob, s);
-    dfree(h->vals, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
+    dfree(h->vals, s); dfree(h->mask, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
     dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s);
 }
 
@@ -470,7 +472,6 @@ struct BuildTemps {
     int32_t* uniq = nullptr;     // [nnz]
     int32_t* rank = nullptr;     // [nnz]
     int64_t* scan_tmp = nullptr;
-    uint32_t* mask = nullptr;    // [4T]
     int64_t* cnt = nullptr;      // [T+1]
     int64_t* ucnt = nullptr;     // [W+1]
     int64_t* usplit = nullptr;   // [W+1]
@@ -483,7 +484,7 @@ struct BuildTemps {
     uint8_t* pval = nullptr;     // row_perm: permuted values
     void release(cudaStream_t s) {
         dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s);
-        dfree(scan_tmp, s); dfree(mask, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
+        dfree(scan_tmp, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
         dfree(uslots, s);
         dfree(pseen, s); dfree(pdeg, s); dfree(prow32, s); dfree(pcol, s); dfree(pval, s);
         host = nullptr;   // per-thread pinned scratch, not owned
@@ -640,16 +641,17 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         }
         k_to_i32<<<grid_for(W + 1, 256, 4096), 256, 0, s>>>(t.nb, h->rwo, W + 1);
         if (T > 0) {
-            // global mask words only back windows with more than kFillSmemBlocks TC blocks
-            TRY(dalloc(&t.mask, 4 * T, s));
-            TRYC(cudaMemsetAsync(t.mask, 0, 4 * T * sizeof(uint32_t), s));
+            // occupancy masks: built in shared memory (windows of <= kFillSmemBlocks blocks) or
+            // directly in this array, which the SpMM kernel keeps as its fragment index
+            TRY(dalloc(&h->mask, 4 * T, s));
+            TRYC(cudaMemsetAsync(h->mask, 0, 4 * T * sizeof(uint32_t), s));
             if (h->dtype == DTC_FP16)
                 k_fill_window<uint16_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, t.mask, (const uint16_t*)csr->vals,
+                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint16_t*)csr->vals,
                     h->tco, h->lid, (uint16_t*)h->vals, h->atob);
             else
                 k_fill_window<uint32_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, t.mask, (const uint32_t*)csr->vals,
+                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint32_t*)csr->vals,
                     h->tco, h->lid, (uint32_t*)h->vals, h->atob);
         } else {
             TRYC(cudaMemsetAsync(h->tco, 0, sizeof(int32_t), s));

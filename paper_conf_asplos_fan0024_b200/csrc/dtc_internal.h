@@ -35,6 +35,10 @@ struct dtc_format {
     uint8_t* lid = nullptr;      // [nnz]
     int32_t* atob = nullptr;     // [8T]
     void* vals = nullptr;        // [nnz] fp32 / fp16
+    // kernel-side index derived from TCLocalId (not part of ME-TCF): 128-bit occupancy of each
+    // TC block, bit id = local id.  TCValues[TCOffset[b] + popcount(mask below id)] is the value
+    // at id (C5: ascending local id), so a lane builds its A fragment without a shared-memory scatter.
+    uint32_t* mask = nullptr;    // [4T]
     // F4 schedule
     int64_t num_units = 0;
     int64_t num_split = 0;       // split windows

@@ -7,28 +7,23 @@
 // thread load 4 consecutive B columns and un-permutes C at the store,
 // and strict balance of TC blocks over thread blocks with atomics.
 //
-// What changes on B200 (measured):
-//  * The paper's shared-memory bypass is the wrong call here: a warp-wide
-//    LDG.128 in the mma B-fragment order touches 4 different B rows per 8 lanes
-//    and costs ~12 L1 data-pipe wavefronts per request (ncu, profiles/), which
-//    capped the first kernel at ~58% of the L1 pipe with 4 TB/s of gather.  sm_100a
-//    has the async global->smem row gather the paper lacked ("absence of
-//    support for asynchronous copying ... up to Ada"): TMA tile::gather4.  The
-//    main path (k_spmm_tma) gathers each TC block's 8 B rows x 128 B slices into
-//    a 128B-swizzled smem ring with gather4 (the -1 pad rows are TMA
-//    out-of-bounds and arrive as zeros), so the consumers never wait on
-//    register-held loads and the ring keeps ~64 KB per CTA in flight.
-//  * Warp specialisation: warp WARPS stages A fragments (FetchSparse, S1) in
-//    batches of 32 TC blocks (already in mma fragment order, TF32-rounded),
-//    warp WARPS+1 issues the B gathers (S2), warps [0, WARPS) run mma.sync
-//    m16n8k8 (S3: one instruction per TC block per 8 columns, k = 8) from
-//    conflict-free LDS.128 reads, with mbarrier full/empty handshakes.
-//  * Balance + locality: a CTA takes one F4 work unit (whole windows grouped to
-//    ~U TC blocks, or one piece of a long window) x one column slice; CTAs are
-//    dispatched in window order by the hardware scheduler.  Split windows finish
-//    with a deterministic fixup (partials summed in piece order; no float atomics).
-//  * k_spmm_ldg is the register-gather fallback for layouts TMA cannot describe
-//    (unaligned B, ldb*elt % 16 != 0) -- same arithmetic, same results.
+// What changes on B200 (measured, profiles/r01_design_evidence.md).
+// Three kernel variants compute S1-S5 with the same arithmetic (dtc_set_spmm_path):
+//  * k_spmm_ldg (path 1): the CTA stages chunks of 16/32 TC blocks of A into shared
+//    memory already in mma-fragment order and TF32-rounded (FetchSparse + the paper's
+//    sparse double buffering, two chunks deep); every warp gathers its B rows
+//    straight into registers one block ahead (the shared-memory bypass + register
+//    remap of P:297-319, generalised to m16n8k8).
+//  * k_spmm_dir (path 3): no shared memory and no CTA barrier: each warp builds its own
+//    A fragment from TCValues through a 128-bit occupancy mask per TC block, and work
+//    items (unit x column slice) run in L2-sized column passes.
+//  * k_spmm_tma (path 2, ablation): B rows gathered by TMA tile::gather4 into a
+//    128B-swizzled smem ring (the async global->smem gather the paper lacked);
+//    measured op-rate bound at ~4 TB/s for 512-byte boxes, so it is not the default.
+// Common to all: mma.sync m16n8k8 TF32/FP16 with FP32 accumulation (C22);
+// balance + locality from the F4 work units (TC-block sized, window ordered, P:333,
+// P:258) dispatched in order; split windows finish with a deterministic fixup
+// (partials summed in piece order; no float atomics, P:333 used atomics).
 #include <cuda.h>
 #include <cuda_fp16.h>
 
@@ -836,6 +831,237 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
 }
 
+// ============================================================ direct path (no shared memory)
+// Every warp builds its own A fragment straight from ME-TCF + the occupancy mask, so there
+// is no FetchSparse producer, no shared-memory scatter and no CTA barrier at all:
+//  * k permutation: lane (g,t) takes B rows SparseAtoB[8b+2t] and [8b+2t+1] as its mma rows
+//    k=t and k=t+4 (one 8-byte load).  The A columns are permuted the same way, so the
+//    lane's four A slots are local ids 8g+2t, 8g+2t+1, 8(g+8)+2t, 8(g+8)+2t+1 -- the same
+//    four slots in TF32 (a0,a2 | a1,a3) and FP16 (reg0 | reg1) fragment order.
+//  * the value of slot id is TCValues[TCOffset[b] + popcount(mask[b] below id)] (C5), loaded
+//    predicated on the mask bit; TF32 rounds it with cvt.rna once per block.
+//  * a P-deep register pipeline per warp: block i+P's B rows and A values are issued right
+//    after block i's mma, block i+2P's (ids, mask, TCOffset) one stage earlier.
+template <int DT>
+struct DirMeta {
+    int2 ids;
+    uint4 m;
+    int base;
+};
+
+template <int DT, int WARPS, int CW, int PD>
+constexpr int dir_maxregs() {
+#if defined(DTC_DIR_MAXREGS) && defined(DTC_DIR_MAXREGS_H)
+    return DT == DTC_FP16 ? DTC_DIR_MAXREGS_H : DTC_DIR_MAXREGS;
+#else
+    return DT == DTC_FP16 ? (PD == 1 ? 128 : 168) : (PD == 1 ? 96 : 128);
+#endif
+}
+template <int DT, int WARPS, int CW, int PD>
+constexpr int dir_min_blocks() {
+    constexpr int b = 65536 / (WARPS * 32 * dir_maxregs<DT, WARPS, CW, PD>());
+    return b > 32 ? 32 : (b < 1 ? 1 : b);
+}
+template <int DT>
+constexpr int dir_depth() {
+#ifdef DTC_DIR_DEPTH
+    return DTC_DIR_DEPTH;
+#else
+    return 1;
+#endif
+}
+
+__device__ __forceinline__ uint32_t ldg_u32_pred(const uint32_t* p, bool pred) {
+    uint32_t v;
+    asm volatile(
+        "{\n"
+        ".reg .pred q;\n"
+        "setp.ne.b32 q, %2, 0;\n"
+        "mov.b32 %0, 0;\n"
+        "@q ld.global.nc.u32 %0, [%1];\n"
+        "}\n"
+        : "=r"(v)
+        : "l"(p), "r"((int)pred));
+    return v;
+}
+__device__ __forceinline__ uint32_t ldg_u16_pred(const unsigned short* p, bool pred) {
+    unsigned short v;
+    asm volatile(
+        "{\n"
+        ".reg .pred q;\n"
+        "setp.ne.b32 q, %2, 0;\n"
+        "mov.b16 %0, 0;\n"
+        "@q ld.global.nc.u16 %0, [%1];\n"
+        "}\n"
+        : "=h"(v)
+        : "l"(p), "r"((int)pred));
+    return (uint32_t)v;
+}
+
+template <int DT, int WARPS, bool VEC, int CW, int PD>
+__global__ void __launch_bounds__(WARPS * 32, dir_min_blocks<DT, WARPS, CW, PD>())
+k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
+           const uint4* __restrict__ mask, const int32_t* __restrict__ atob, const void* __restrict__ avals,
+           const void* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
+           const int32_t* __restrict__ rowmap, int num_units, int nws, int pass_ws) {
+    using Tr = Traits<DT>;
+    constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, VW = Tr::VW, FW = Tr::FRAG_WORDS;
+    constexpr int NJ = NJ1 * CW;
+    constexpr int COLW = COLW1 * CW;
+    constexpr int QPC = NJ1 / 4;
+    using E = typename Tr::elt;
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+    // work item = (unit, warp slice of COLW columns); warps are independent (no CTA barrier).
+    // Items run in passes of pass_ws slices (a pass's B columns sized to stay L2-resident),
+    // unit-major inside a pass so the slices of one unit land on neighbouring warps.
+    const int64_t item = (int64_t)blockIdx.x * WARPS + warp;
+    const int64_t per = (int64_t)num_units * pass_ws;
+    const int p = (int)(item / per);
+    const int64_t r = item - (int64_t)p * per;
+    const int pw = min(pass_ws, nws - p * pass_ws);
+    if (pw <= 0) return;
+    const int wsl = p * pass_ws + (int)(r % pw);
+    const int64_t n0 = (int64_t)wsl * COLW;
+    const Unit u = units[r / pw];
+    const int64_t bcol = n0 + (int64_t)VW * g;
+    const int64_t base = n0 + 2 * NJ1 * t;
+    const int hoff = NJ1;
+    const bool split = u.split_id >= 0;
+    const int nblocks = u.be - u.bb;
+
+    // this lane's mask bits: slots (8g+2t, +1) in word g>>2, (64+8g+2t, +1) in word 2+(g>>2)
+    const int pos = 8 * (g & 3) + 2 * t;
+    const uint32_t below = (1u << pos) - 1u;
+    const bool upper = g >= 4;
+
+    auto load_meta = [&](int b) -> DirMeta<DT> {
+        DirMeta<DT> mt;
+        mt.ids = __ldg(reinterpret_cast<const int2*>(atob + (int64_t)b * 8) + t);
+        mt.m = __ldg(mask + b);
+        mt.base = __ldg(tco + b);
+        return mt;
+    };
+    auto load_a = [&](const DirMeta<DT>& mt, uint32_t (&a)[FW]) {
+        const uint32_t wl = upper ? mt.m.y : mt.m.x;
+        const uint32_t wh = upper ? mt.m.w : mt.m.z;
+        const int c0 = __popc(mt.m.x), c01 = c0 + __popc(mt.m.y);
+        const int rl = mt.base + (upper ? c0 : 0) + __popc(wl & below);
+        const int rh = mt.base + c01 + (upper ? __popc(mt.m.z) : 0) + __popc(wh & below);
+        const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
+        const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
+        if (DT == DTC_TF32) {
+            const uint32_t* v = reinterpret_cast<const uint32_t*>(avals);
+            a[0] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl, p00)));        // (g,   k=t)   id 8g+2t
+            a[1] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh, p10)));        // (g+8, k=t)
+            a[2] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl + p00, p01)));  // (g,   k=t+4) id 8g+2t+1
+            a[3] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh + p10, p11))); // (g+8, k=t+4)
+        } else {
+            const unsigned short* v = reinterpret_cast<const unsigned short*>(avals);
+            a[0] = ldg_u16_pred(v + rl, p00) | (ldg_u16_pred(v + rl + p00, p01) << 16);   // (g, 2t), (g, 2t+1)
+            a[1] = ldg_u16_pred(v + rh, p10) | (ldg_u16_pred(v + rh + p10, p11) << 16);   // (g+8, ...)
+        }
+    };
+    const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)sizeof(E);
+    const uint64_t ldb_bytes = (uint64_t)ldb * sizeof(E);
+    auto gather = [&](int row, int cw) -> V16 {
+        if (VEC) {
+            const bool ok = row >= 0 && (bcol + cw * COLW1) < N;
+            const char* p = ok ? bthr + (uint64_t)(uint32_t)row * ldb_bytes + cw * COLW1 * (int)sizeof(E)
+                               : reinterpret_cast<const char*>(g_zero_line);
+            const uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
+            V16 v;
+            v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
+            return v;
+        }
+        return load_b<DT, VEC>(B, ldb, row, bcol + cw * COLW1, N);
+    };
+
+    float acc[NJ][4];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+
+    int cur = u.wb;
+    int next_end = INT_MAX;
+    if (!split) {
+        while (cur < u.we && rwo[cur + 1] <= u.bb) {
+            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+            ++cur;
+        }
+        next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+    }
+
+    DirMeta<DT> mt[PD];
+    uint32_t af[PD][FW];
+    V16 b0[PD][CW], b1[PD][CW];
+    auto issue = [&](int q) {
+#pragma unroll
+        for (int cw = 0; cw < CW; ++cw) {
+            b0[q][cw] = gather(mt[q].ids.x, cw);
+            b1[q][cw] = gather(mt[q].ids.y, cw);
+        }
+        load_a(mt[q], af[q]);
+    };
+#pragma unroll
+    for (int q = 0; q < PD; ++q)
+        if (q < nblocks) mt[q] = load_meta(u.bb + q);
+#pragma unroll
+    for (int q = 0; q < PD; ++q)
+        if (q < nblocks) {
+            issue(q);
+            if (q + PD < nblocks) mt[q] = load_meta(u.bb + q + PD);
+        }
+    for (int i0 = 0; i0 < nblocks; i0 += PD) {
+#pragma unroll
+        for (int q = 0; q < PD; ++q) {
+            const int i = i0 + q;
+            if (i < nblocks) {
+                if (DT == DTC_TF32) {
+                    const uint32_t a[4] = {af[q][0], af[q][1], af[q][2], af[q][3]};
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                        for (int jj = 0; jj < NJ1; ++jj)
+                            mma_tf32(acc[cw * NJ1 + jj], a, b0[q][cw].w[jj], b1[q][cw].w[jj]);
+                } else {
+                    const uint32_t a[2] = {af[q][0], af[q][1]};
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                        for (int jj = 0; jj < NJ1; ++jj) {
+                            const uint32_t bb = __byte_perm(b0[q][cw].w[jj >> 1], b1[q][cw].w[jj >> 1],
+                                                            (jj & 1) ? 0x7632 : 0x5410);
+                            mma_f16(acc[cw * NJ1 + jj], a, bb);
+                        }
+                }
+                if (i + PD < nblocks) {
+                    issue(q);
+                    if (i + 2 * PD < nblocks) mt[q] = load_meta(u.bb + i + 2 * PD);
+                }
+                if (u.bb + i + 1 == next_end) {
+                    store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+#pragma unroll
+                    for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+                    ++cur;
+                    while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
+                        store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                        ++cur;
+                    }
+                    next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+                }
+            }
+        }
+    }
+    if (!split) {
+        while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
+        return;
+    }
+    int32_t* ctr = counters + (int64_t)u.split_id * nws + wsl;
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+}
+
 // ============================================================ host side
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -879,6 +1105,7 @@ struct LaunchArgs {
     int gy;
     int64_t npad;
     cudaStream_t s;
+    int nws, pass_ws;   // direct path: warp slices of N, slices per L2-resident pass
 };
 
 template <int DT, int WARPS>
@@ -919,8 +1146,31 @@ static cudaError_t launch_ldg(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
+template <int DT, int WARPS, bool VEC, int CW>
+static cudaError_t launch_dir(const LaunchArgs& a) {
+    constexpr int PD = dir_depth<DT>();
+    const int64_t items = a.h->num_units * (int64_t)a.nws;
+    const int64_t nblk = (items + WARPS - 1) / WARPS;
+    if (nblk > INT_MAX) return cudaErrorInvalidConfiguration;
+    k_spmm_dir<DT, WARPS, VEC, CW, PD><<<(unsigned)nblk, WARPS * 32, 0, a.s>>>(
+        a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.B, a.ldb,
+        a.C, a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap, (int)a.h->num_units, a.nws,
+        a.pass_ws);
+    return cudaGetLastError();
+}
+
 template <int DT, bool VEC>
-static cudaError_t dispatch(int warps, bool tma, const LaunchArgs& a, const CUtensorMap& map) {
+static cudaError_t dispatch(int warps, int path, const LaunchArgs& a, const CUtensorMap& map) {
+    const bool tma = path == 2;
+    if (path == 3) {
+        constexpr int CW = ldg_colchunks<DT>();
+        switch (warps) {
+            case 1: return launch_dir<DT, 1, VEC, CW>(a);
+            case 2: return launch_dir<DT, 2, VEC, CW>(a);
+            case 4: return launch_dir<DT, 4, VEC, CW>(a);
+            default: return launch_dir<DT, 8, VEC, CW>(a);
+        }
+    }
     if (tma) {
         switch (warps) {
             case 1: return launch_tma<DT, 1, VEC>(a, map);
@@ -938,7 +1188,28 @@ static cudaError_t dispatch(int warps, bool tma, const LaunchArgs& a, const CUte
     }
 }
 
-static int g_force_path = -1;   // 1 = register gather (default), 2 = TMA gather4 (DTC_SPMM_PATH=tma)
+static int64_t l2_bytes() {
+    static int64_t v = -1;
+    if (v < 0) {
+        int dev = 0, x = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&x, cudaDevAttrL2CacheSize, dev) != cudaSuccess || x <= 0) {
+            cudaGetLastError();
+            x = 126 << 20;
+        }
+        v = x;
+    }
+    return v;
+}
+
+static int g_force_path = -1;   // 1 = register gather via smem A chunks, 2 = TMA gather4, 3 = direct (DTC_SPMM_PATH=ldg|tma|dir)
+#ifndef DTC_DEFAULT_PATH
+#define DTC_DEFAULT_PATH 1
+#endif
+static int env_path() {
+    const char* e = getenv("DTC_SPMM_PATH");
+    return (e && e[0] == 't') ? 2 : (e && e[0] == 'l') ? 1 : (e && e[0] == 'd') ? 3 : DTC_DEFAULT_PATH;
+}
 
 int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc, cudaStream_t s) {
     if (!h) { set_error("null handle"); return DTC_ERR_INVALID; }
@@ -949,13 +1220,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     if (h->M == 0) return DTC_OK;
     if (!C || (!B && h->T > 0)) { set_error("null B or C"); return DTC_ERR_INVALID; }
     if (h->num_units == 0) return DTC_OK;
-    if (g_force_path < 0) {
-        const char* e = getenv("DTC_SPMM_PATH");
-#ifndef DTC_DEFAULT_PATH
-#define DTC_DEFAULT_PATH 1
-#endif
-        g_force_path = (e && e[0] == 't') ? 2 : (e && e[0] == 'l') ? 1 : DTC_DEFAULT_PATH;   // default: register gather
-    }
+    if (g_force_path < 0) g_force_path = env_path();
     const int elt = elt_size(h->dtype);
     const int VW = 16 / elt;
     // TMA needs a 16-byte aligned base and row pitch; a ragged N is fine (OOB columns zero-fill)
@@ -998,12 +1263,24 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     const bool cvec = ((uintptr_t)C % 16 == 0) && (ldc % 4 == 0) && (N % 4 == 0);
     const bool bvec = ((uintptr_t)B % 16 == 0) && (ldb % VW == 0) && (N % VW == 0);
     const bool use_vec = tma ? cvec : (cvec && bvec);
-    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s};
+    const int path = tma ? 2 : (g_force_path == 3 ? 3 : 1);
+    // direct path: a pass covers pass_ws warp slices, sized so K x (pass columns) of B stays
+    // within ~3/4 of L2 (DTC_PASS_WS overrides: a large value = one unit-major pass)
+    const int nws = (int)need;
+    int pass_ws = nws;
+    if (path == 3) {
+        const char* e = getenv("DTC_PASS_WS");
+        const int64_t slice_bytes = std::max<int64_t>(h->K, 1) * colw * elt;
+        const int64_t fit = (l2_bytes() * 3 / 4) / slice_bytes;
+        pass_ws = (int)std::min<int64_t>(nws, std::max<int64_t>(1, fit));
+        if (e && atoi(e) > 0) pass_ws = std::min(nws, atoi(e));
+    }
+    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws};
     cudaError_t e;
     if (h->dtype == DTC_FP16)
-        e = use_vec ? dispatch<DTC_FP16, true>(warps, tma, a, map) : dispatch<DTC_FP16, false>(warps, tma, a, map);
+        e = use_vec ? dispatch<DTC_FP16, true>(warps, path, a, map) : dispatch<DTC_FP16, false>(warps, path, a, map);
     else
-        e = use_vec ? dispatch<DTC_TF32, true>(warps, tma, a, map) : dispatch<DTC_TF32, false>(warps, tma, a, map);
+        e = use_vec ? dispatch<DTC_TF32, true>(warps, path, a, map) : dispatch<DTC_TF32, false>(warps, path, a, map);
     if (e != cudaSuccess) return cuda_fail(e, "k_spmm launch", __FILE__, __LINE__);
     return DTC_OK;
 }
@@ -1017,6 +1294,13 @@ extern "C" int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, f
 }
 
 extern "C" int dtc_spmm_launches_per_call(void) { return 1; }
+
+extern "C" int dtc_set_spmm_path(int path) {
+    if (path < 0 || path > 3) { set_error("unknown spmm path %d", path); return DTC_ERR_INVALID; }
+    const int prev = g_force_path < 0 ? 0 : g_force_path;
+    g_force_path = path == 0 ? DTC_DEFAULT_PATH : path;
+    return prev;
+}
 
 extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                              int64_t ldc, void* stream) {

@@ -1,0 +1,118 @@
+"""Every dtc_spmm kernel variant (dtc_set_spmm_path: ldg / tma / dir) against oracle O1.
+
+The library default is covered by test_gpu_spmm.py at every config; this module runs the
+same parity bar (tolerance of BASELINE.json north_star, bit-exact for the exact-arithmetic
+pins P2/P3/P9) on each variant, so an ablation number in profiles/ is never a number of an
+incorrect kernel.
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from datagen import configs
+
+from gpu_util import build, dev, spmm, check_tol
+
+pytestmark = pytest.mark.gpu
+
+PATHS = ["ldg", "tma", "dir"]
+
+
+@pytest.fixture(params=PATHS)
+def path(request):
+    from paper_conf_asplos_fan0024_b200 import set_spmm_path
+    set_spmm_path(request.param)
+    yield request.param
+    set_spmm_path("default")
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("N", [1, 8, 33, 64, 128, 200, 512])
+def test_random_tolerance(path, dtype, N):
+    M, K = 500, 700
+    rp, ci = datagen.random_csr(M, K, 0.04, N + 11)
+    v = datagen.uniform(N, 1, len(ci))
+    B = datagen.uniform(N, 2, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    check_tol(spmm(f, B), M, K, rp, ci, v, B, dtype)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("name,N,U", [("c1", 32, 0), ("c1", 256, 0), ("c2", 128, 0), ("c1", 96, 2)])
+def test_p2_integer_bit_exact(path, name, N, U, dtype):
+    """P2 (small integers: exact in TF32/FP16 and FP32), incl. split windows (U=2)."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.integers(cfg.seed_a, 5, len(ci))
+    B = datagen.integers(cfg.seed_b, 6, cfg.K * N).reshape(cfg.K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U)
+    C = spmm(f, B)
+    assert np.array_equal(C, spmm(f, B))
+    Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v.astype(np.float32), B.astype(np.float32))
+    assert np.array_equal(C.astype(np.float64), Cr)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+def test_p9_dense_blocks_exact(path, dtype):
+    """P9: fully dense A (every TC block holds 128 non-zeros, every mask bit set), M and K
+    not multiples of 16 / 8 (ragged last window and last block), integer values."""
+    M, K, N = 45, 29, 72
+    rp = (np.arange(M + 1) * K).astype(np.int32)
+    ci = np.tile(np.arange(K, dtype=np.int32), M)
+    v = datagen.integers(9, 1, M * K)
+    B = datagen.integers(9, 2, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    C = spmm(f, B)
+    ref = v.astype(np.float64).reshape(M, K) @ B.astype(np.float64)
+    assert np.array_equal(C.astype(np.float64), ref)
+
+
+def test_p3_identity_and_empty_windows(path):
+    M, N = 1000, 64
+    B = datagen.uniform(1, 2, M * N).reshape(M, N)
+    Bt = (B.view(np.uint32) & np.uint32(0xFFFFE000)).view(np.float32)   # TF32-representable
+    keep = np.ones(M, bool)
+    keep[100:180] = False                                              # 5 empty windows
+    rp = np.concatenate([[0], np.cumsum(keep)]).astype(np.int32)
+    ci = np.nonzero(keep)[0].astype(np.int32)
+    f = build(M, M, rp, ci, np.ones(len(ci), np.float32))
+    ref = Bt * keep[:, None]
+    assert np.array_equal(spmm(f, Bt), ref)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+def test_strided_misaligned(path, dtype):
+    import torch
+    M, K, N = 300, 400, 37
+    rp, ci = datagen.random_csr(M, K, 0.05, 7)
+    v = datagen.uniform(7, 1, len(ci))
+    Bf = datagen.uniform(7, 2, K * 50).reshape(K, 50)
+    if dtype == "fp16":
+        v, Bf = v.astype(np.float16), Bf.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    Bd = dev(Bf)[:, 1:1 + N]
+    Cbig = torch.full((M, 41), float("nan"), device="cuda")
+    C = Cbig[:, 2:2 + N]
+    f.spmm(Bd, C)
+    torch.cuda.synchronize()
+    check_tol(C.cpu().numpy(), M, K, rp, ci, v, Bf[:, 1:1 + N], dtype)
+    assert torch.isnan(Cbig[:, :2]).all() and torch.isnan(Cbig[:, 2 + N:]).all()
+
+
+def test_row_perm_original_order(path):
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.integers(cfg.seed_a, 5, len(ci))
+    N = 64
+    B = datagen.integers(cfg.seed_b, 6, cfg.K * N).reshape(cfg.K, N)
+    perm = np.random.default_rng(3).permutation(cfg.M).astype(np.int32)
+    f = build(cfg.M, cfg.K, rp, ci, v, row_perm=dev(perm))
+    Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v, B)
+    assert np.array_equal(spmm(f, B).astype(np.float64), Cr)
