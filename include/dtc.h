@@ -143,9 +143,10 @@ int dtc_spmm_launches_per_call(void);
  *   0 = library default, 1 = register gather with shared-memory A chunks (the paper's
  *   FetchSparse/SDB structure), 2 = TMA tile::gather4 B ring,
  *   3 = direct: each warp builds its A fragment from TCValues via the per-block
- *   occupancy mask (no shared memory, no CTA barrier).
+ *   occupancy mask (no shared memory, no CTA barrier), 4 = TMA gather4 of whole
+ *   512-byte row slices into 528-byte padded smem rows (conflict-free fragment reads).
  * Process-wide, takes effect at the next dtc_spmm; the environment variable
- * DTC_SPMM_PATH=ldg|tma|dir sets the initial value.  Returns the previous setting
+ * DTC_SPMM_PATH=ldg|tma|dir|pad sets the initial value.  Returns the previous setting
  * (0 if it was the default), or DTC_ERR_INVALID for an unknown path. */
 int dtc_set_spmm_path(int path);
 

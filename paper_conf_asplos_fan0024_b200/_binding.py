@@ -123,7 +123,7 @@ def launches_per_call() -> int:
     return int(lib().dtc_spmm_launches_per_call())
 
 
-SPMM_PATHS = {"default": 0, "ldg": 1, "tma": 2, "dir": 3}
+SPMM_PATHS = {"default": 0, "ldg": 1, "tma": 2, "dir": 3, "pad": 4}
 
 
 def set_spmm_path(path) -> int:

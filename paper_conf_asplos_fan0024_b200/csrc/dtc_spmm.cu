@@ -898,6 +898,41 @@ __device__ __forceinline__ uint32_t ldg_u16_pred(const unsigned short* p, bool p
     return (uint32_t)v;
 }
 
+// (ids, mask, TCOffset) of TC block b for lane t: B rows SparseAtoB[8b+2t], [8b+2t+1]
+template <int DT>
+__device__ __forceinline__ DirMeta<DT> dir_load_meta(int b, int t, const int32_t* __restrict__ atob,
+                                                     const uint4* __restrict__ mask, const int32_t* __restrict__ tco) {
+    DirMeta<DT> mt;
+    mt.ids = __ldg(reinterpret_cast<const int2*>(atob + (int64_t)b * 8) + t);
+    mt.m = __ldg(mask + b);
+    mt.base = __ldg(tco + b);
+    return mt;
+}
+// A fragment of one TC block for lane (g,t) under the k permutation (slots 8g+2t, 8g+2t+1,
+// 8(g+8)+2t, 8(g+8)+2t+1): value rank = popcount of the mask below the slot (C5)
+template <int DT>
+__device__ __forceinline__ void dir_load_a(const DirMeta<DT>& mt, uint32_t (&a)[Traits<DT>::FRAG_WORDS], int pos,
+                                           uint32_t below, bool upper, const void* __restrict__ avals) {
+    const uint32_t wl = upper ? mt.m.y : mt.m.x;
+    const uint32_t wh = upper ? mt.m.w : mt.m.z;
+    const int c0 = __popc(mt.m.x), c01 = c0 + __popc(mt.m.y);
+    const int rl = mt.base + (upper ? c0 : 0) + __popc(wl & below);
+    const int rh = mt.base + c01 + (upper ? __popc(mt.m.z) : 0) + __popc(wh & below);
+    const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
+    const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
+    if (DT == DTC_TF32) {
+        const uint32_t* v = reinterpret_cast<const uint32_t*>(avals);
+        a[0] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl, p00)));        // (g,   k=t)   id 8g+2t
+        a[1] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh, p10)));        // (g+8, k=t)
+        a[2] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl + p00, p01)));  // (g,   k=t+4) id 8g+2t+1
+        a[3] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh + p10, p11)));  // (g+8, k=t+4)
+    } else {
+        const unsigned short* v = reinterpret_cast<const unsigned short*>(avals);
+        a[0] = ldg_u16_pred(v + rl, p00) | (ldg_u16_pred(v + rl + p00, p01) << 16);   // (g, 2t), (g, 2t+1)
+        a[1] = ldg_u16_pred(v + rh, p10) | (ldg_u16_pred(v + rh + p10, p11) << 16);   // (g+8, ...)
+    }
+}
+
 template <int DT, int WARPS, bool VEC, int CW, int PD>
 __global__ void __launch_bounds__(WARPS * 32, dir_min_blocks<DT, WARPS, CW, PD>())
 k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, const int32_t* __restrict__ tco,
@@ -937,33 +972,8 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     const uint32_t below = (1u << pos) - 1u;
     const bool upper = g >= 4;
 
-    auto load_meta = [&](int b) -> DirMeta<DT> {
-        DirMeta<DT> mt;
-        mt.ids = __ldg(reinterpret_cast<const int2*>(atob + (int64_t)b * 8) + t);
-        mt.m = __ldg(mask + b);
-        mt.base = __ldg(tco + b);
-        return mt;
-    };
-    auto load_a = [&](const DirMeta<DT>& mt, uint32_t (&a)[FW]) {
-        const uint32_t wl = upper ? mt.m.y : mt.m.x;
-        const uint32_t wh = upper ? mt.m.w : mt.m.z;
-        const int c0 = __popc(mt.m.x), c01 = c0 + __popc(mt.m.y);
-        const int rl = mt.base + (upper ? c0 : 0) + __popc(wl & below);
-        const int rh = mt.base + c01 + (upper ? __popc(mt.m.z) : 0) + __popc(wh & below);
-        const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
-        const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
-        if (DT == DTC_TF32) {
-            const uint32_t* v = reinterpret_cast<const uint32_t*>(avals);
-            a[0] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl, p00)));        // (g,   k=t)   id 8g+2t
-            a[1] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh, p10)));        // (g+8, k=t)
-            a[2] = to_tf32(__uint_as_float(ldg_u32_pred(v + rl + p00, p01)));  // (g,   k=t+4) id 8g+2t+1
-            a[3] = to_tf32(__uint_as_float(ldg_u32_pred(v + rh + p10, p11))); // (g+8, k=t+4)
-        } else {
-            const unsigned short* v = reinterpret_cast<const unsigned short*>(avals);
-            a[0] = ldg_u16_pred(v + rl, p00) | (ldg_u16_pred(v + rl + p00, p01) << 16);   // (g, 2t), (g, 2t+1)
-            a[1] = ldg_u16_pred(v + rh, p10) | (ldg_u16_pred(v + rh + p10, p11) << 16);   // (g+8, ...)
-        }
-    };
+    auto load_meta = [&](int b) -> DirMeta<DT> { return dir_load_meta<DT>(b, t, atob, mask, tco); };
+    auto load_a = [&](const DirMeta<DT>& mt, uint32_t (&a)[FW]) { dir_load_a<DT>(mt, a, pos, below, upper, avals); };
     const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)sizeof(E);
     const uint64_t ldb_bytes = (uint64_t)ldb * sizeof(E);
     auto gather = [&](int row, int cw) -> V16 {
@@ -1062,6 +1072,196 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
     split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
 }
 
+// ============================================================ TMA path with padded rows (path 4)
+// B rows arrive by TMA tile::gather4 in boxes of one 512-byte column slice plus 16 bytes of
+// padding (128 fp32 / 256 fp16 columns + 4 / 8 extra), so consecutive rows of a stage sit
+// 528 bytes apart: 528 = 16 (mod 128) shifts each row by one 16-byte bank group and the
+// fragment reads (lane (g,t): rows 2t and 2t+1, 16-byte chunk g of a 128-byte segment) hit 8
+// distinct bank groups per 8-lane phase -- conflict-free without a swizzle, and 4x fewer TMA
+// ops per byte than 128-byte swizzled boxes (the r01 gather4 ablation was op-rate bound).
+// The gather moves no data through the LSU pipe (the register gather's limiter, ncu
+// l1tex data-pipe 85%); one producer warp runs up to kPadStages blocks ahead.
+// Consumer warps: 2 per slice, each owning 2 x 128-byte segments (64 fp32 / 128 fp16 columns),
+// A fragments built in registers from the occupancy mask one block ahead (as k_spmm_dir).
+constexpr int kPadBoxElts = 132;                 // 4-byte elements per box row (128 + 4 pad)
+constexpr int kPadRowBytes = kPadBoxElts * 4;    // 528
+constexpr int kPadSliceBytes = 8 * kPadRowBytes; // one TC block x one slice
+template <int SL>
+constexpr int pad_stages() {
+#ifdef DTC_PAD_STAGES
+    return DTC_PAD_STAGES;
+#else
+    return SL == 1 ? 12 : (SL == 2 ? 6 : 3);
+#endif
+}
+template <int SL>
+constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * kPadSliceBytes + 128; }
+template <int DT, int SL>
+constexpr int pad_maxregs() {
+#ifdef DTC_PAD_MAXREGS
+    return DTC_PAD_MAXREGS;
+#else
+    return DT == DTC_FP16 ? 128 : 104;
+#endif
+}
+
+template <int DT, int SL, bool VEC>
+__global__ void __launch_bounds__((2 * SL + 1) * 32, 65536 / ((2 * SL + 1) * 32 * pad_maxregs<DT, SL>()))
+k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
+           const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
+           const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
+           float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
+           const int32_t* __restrict__ rowmap) {
+    using Tr = Traits<DT>;
+    constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
+    constexpr int CW = 2;                      // 128-byte segments per consumer warp
+    constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;
+    constexpr int R = pad_stages<SL>();
+    constexpr int STAGE = SL * kPadSliceBytes;
+    constexpr int SLICE_COLS = 4 * COLW1;      // 128 fp32 / 256 fp16 columns per slice
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t* ring = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 127) & ~uintptr_t(127));
+    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R];
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const Unit u = units[blockIdx.x];
+    const int64_t col0 = (int64_t)blockIdx.y * SL * SLICE_COLS;          // first C column of the CTA
+    const int64_t nsl64 = (N - col0 + SLICE_COLS - 1) / SLICE_COLS;
+    const int nsl = nsl64 < SL ? (int)nsl64 : SL;
+    const int ncons = 2 * nsl;
+    const int nblocks = u.be - u.bb;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < R; ++i) {
+            mbar_init(&bar_full[i], 1);
+            mbar_init(&bar_empty[i], ncons);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (warp == 2 * SL) {
+        // ================= producer: gather4 of 4 B rows x one slice per op =================
+        const uint32_t tx = (uint32_t)nsl * kPadSliceBytes;
+        const int half = lane & 1, jl = lane >> 1;     // lane holds rows 4*half.. of block i0 + jl
+        const int32_t tcol = (int32_t)(col0 * (int64_t)sizeof(typename Tr::elt) / 4);   // 4-byte TMA columns
+        auto ids_of = [&](int i0) -> int4 {
+            const int i = i0 + jl;
+            return i < nblocks ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(u.bb + i) * 8) + half)
+                               : make_int4(-1, -1, -1, -1);
+        };
+        int4 cur = ids_of(0);
+        for (int i0 = 0; i0 < nblocks; i0 += 16) {
+            const int4 nxt = (i0 + 16 < nblocks) ? ids_of(i0 + 16) : make_int4(-1, -1, -1, -1);
+            const int nj = min(16, nblocks - i0);
+            for (int j = 0; j < nj; ++j) {
+                const int i = i0 + j, s = i % R;
+                if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
+                if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
+                __syncwarp();
+                if (jl == j) {
+                    for (int sl = 0; sl < nsl; ++sl) {
+                        const uint32_t dst = smem_u32(ring + s * STAGE + sl * kPadSliceBytes + half * 4 * kPadRowBytes);
+                        asm volatile(
+                            "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+                            " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
+                            "l"(&bmap), "r"(tcol + sl * 128), "r"(cur.x), "r"(cur.y), "r"(cur.z), "r"(cur.w),
+                            "r"(smem_u32(&bar_full[s]))
+                            : "memory");
+                    }
+                }
+                __syncwarp();
+            }
+            cur = nxt;
+        }
+        return;
+    }
+    if (warp >= ncons) return;
+
+    // ================= consumers (S1 A fragments, S3 mma, S4/S5) =================
+    const int g = lane >> 2, t = lane & 3;
+    const int sl = warp >> 1;                            // slice of this warp
+    const int64_t n0 = col0 + (int64_t)warp * CW * COLW1;
+    const int64_t base = n0 + 2 * NJ1 * t;
+    const int hoff = NJ1;
+    const bool split = u.split_id >= 0;
+    const int pos = 8 * (g & 3) + 2 * t;
+    const uint32_t below = (1u << pos) - 1u;
+    const bool upper = g >= 4;
+    // smem byte offsets of the thread's rows 2t / 2t+1 at 16-byte chunk g of the warp's first segment
+    const int roff0 = sl * kPadSliceBytes + (2 * t) * kPadRowBytes + (warp & 1) * CW * 128 + g * 16;
+    const int roff1 = roff0 + kPadRowBytes;
+
+    float acc[NJ][4];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+    int cur = u.wb;
+    int next_end = INT_MAX;
+    if (!split) {
+        while (cur < u.we && rwo[cur + 1] <= u.bb) {
+            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+            ++cur;
+        }
+        next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+    }
+    DirMeta<DT> mt;
+    uint32_t af[FW];
+    if (nblocks > 0) {
+        mt = dir_load_meta<DT>(u.bb, t, atob, mask, tco);
+        dir_load_a<DT>(mt, af, pos, below, upper, avals);
+        if (nblocks > 1) mt = dir_load_meta<DT>(u.bb + 1, t, atob, mask, tco);
+    }
+    for (int i = 0; i < nblocks; ++i) {
+        const int s = i % R;
+        uint32_t a[FW];
+#pragma unroll
+        for (int k = 0; k < FW; ++k) a[k] = af[k];
+        if (i + 1 < nblocks) {
+            dir_load_a<DT>(mt, af, pos, below, upper, avals);
+            if (i + 2 < nblocks) mt = dir_load_meta<DT>(u.bb + i + 2, t, atob, mask, tco);
+        }
+        mbar_wait(&bar_full[s], (i / R) & 1);
+        const uint8_t* st = ring + s * STAGE;
+#pragma unroll
+        for (int cw = 0; cw < CW; ++cw) {
+            const uint4 x0 = *reinterpret_cast<const uint4*>(st + roff0 + cw * 128);
+            const uint4 x1 = *reinterpret_cast<const uint4*>(st + roff1 + cw * 128);
+            const uint32_t y0[4] = {x0.x, x0.y, x0.z, x0.w};
+            const uint32_t y1[4] = {x1.x, x1.y, x1.z, x1.w};
+            if constexpr (DT == DTC_TF32) {
+                const uint32_t aa[4] = {a[0], a[1], a[2], a[3]};
+#pragma unroll
+                for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[cw * NJ1 + jj], aa, y0[jj & 3], y1[jj & 3]);
+            } else {
+                const uint32_t aa[2] = {a[0], a[1]};
+#pragma unroll
+                for (int jj = 0; jj < NJ1; ++jj) {
+                    const uint32_t bb = __byte_perm(y0[(jj >> 1) & 3], y1[(jj >> 1) & 3], (jj & 1) ? 0x7632 : 0x5410);
+                    mma_f16(acc[cw * NJ1 + jj], aa, bb);
+                }
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&bar_empty[s]);
+        if (u.bb + i + 1 == next_end) {
+            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+#pragma unroll
+            for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+            ++cur;
+            while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
+                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                ++cur;
+            }
+            next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+        }
+    }
+    if (!split) {
+        while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
+        return;
+    }
+    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+}
+
 // ============================================================ host side
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -1093,6 +1293,22 @@ static bool make_bmap(CUtensorMap* map, const void* B, int64_t K, int64_t N, int
     CUresult r = enc(map, dtype == DTC_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
                      const_cast<void*>(B), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                      CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+// Tensor map of B viewed as 4-byte elements (fp16 pairs for FP16): K rows x N*elt/4 columns,
+// gather4 boxes of kPadBoxElts x 1, no swizzle (rows land 528 bytes apart, see k_spmm_pad).
+static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype) {
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return false;
+    const int elt = elt_size(dtype);
+    cuuint64_t dims[2] = {(cuuint64_t)(N * elt / 4), (cuuint64_t)K};
+    cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
+    cuuint32_t box[2] = {(cuuint32_t)kPadBoxElts, 1};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(B), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
 
@@ -1159,8 +1375,30 @@ static cudaError_t launch_dir(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
+template <int DT, int SL, bool VEC>
+static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
+    const size_t smem = pad_smem_bytes<SL>();
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_spmm_pad<DT, SL, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr = true;
+    }
+    dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
+    k_spmm_pad<DT, SL, VEC><<<grid, (2 * SL + 1) * 32, smem, a.s>>>(
+        map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
+        a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap);
+    return cudaGetLastError();
+}
+
 template <int DT, bool VEC>
 static cudaError_t dispatch(int warps, int path, const LaunchArgs& a, const CUtensorMap& map) {
+    if (path == 4) {
+        switch (warps) {   // warps = slices per CTA here
+            case 1: return launch_pad<DT, 1, VEC>(a, map);
+            case 2: return launch_pad<DT, 2, VEC>(a, map);
+            default: return launch_pad<DT, 4, VEC>(a, map);
+        }
+    }
     const bool tma = path == 2;
     if (path == 3) {
         constexpr int CW = ldg_colchunks<DT>();
@@ -1208,7 +1446,8 @@ static int g_force_path = -1;   // 1 = register gather via smem A chunks, 2 = TM
 #endif
 static int env_path() {
     const char* e = getenv("DTC_SPMM_PATH");
-    return (e && e[0] == 't') ? 2 : (e && e[0] == 'l') ? 1 : (e && e[0] == 'd') ? 3 : DTC_DEFAULT_PATH;
+    return (e && e[0] == 't') ? 2 : (e && e[0] == 'l') ? 1 : (e && e[0] == 'd') ? 3 : (e && e[0] == 'p') ? 4
+                                                                                                 : DTC_DEFAULT_PATH;
 }
 
 int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc, cudaStream_t s) {
@@ -1226,20 +1465,32 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     // TMA needs a 16-byte aligned base and row pitch; a ragged N is fine (OOB columns zero-fill)
     CUtensorMap map;
     memset(&map, 0, sizeof(map));
-    bool tma = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && h->K < (int64_t(1) << 31) &&
-               N < (int64_t(1) << 31) && g_force_path == 2;
-    if (tma) tma = make_bmap(&map, B, h->K, N, ldb, h->dtype);
-    // columns per warp: the TMA path uses one 128-byte slice per warp, the register path CW slices
+    const bool tma_ok = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) &&
+                        h->K < (int64_t(1) << 31) && N < (int64_t(1) << 31);
+    int path = g_force_path == 3 ? 3 : 1;
+    if (g_force_path == 2 && tma_ok && make_bmap(&map, B, h->K, N, ldb, h->dtype)) path = 2;
+    if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype)) path = 4;
+    // columns per warp: the 128B-swizzled TMA path one 128-byte slice per warp, the others two
     const int colw_tma = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
     const int colw_ldg = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW * ldg_colchunks<DTC_FP16>()
                                                : Traits<DTC_TF32>::COLW * ldg_colchunks<DTC_TF32>();
-    const int colw = tma ? colw_tma : colw_ldg;
+    const int colw = path == 2 ? colw_tma : colw_ldg;
     const int64_t need = (N + colw - 1) / colw;
-    const int warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
-    const int64_t gy64 = (N + (int64_t)warps * colw - 1) / ((int64_t)warps * colw);
+    int warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
+    int64_t cta_cols = (int64_t)warps * colw;
+    if (path == 4) {
+        // warps := slices (of 512 bytes of a B row) per CTA; two consumer warps per slice
+        const int64_t slice_cols = 512 / elt;
+        const int64_t nsl = (N + slice_cols - 1) / slice_cols;
+        const char* e = getenv("DTC_PAD_SL");
+        const int slmax = (e && atoi(e) > 0) ? atoi(e) : 2;
+        warps = nsl >= 4 && slmax >= 4 ? 4 : (nsl >= 2 && slmax >= 2 ? 2 : 1);
+        cta_cols = warps * slice_cols;
+    }
+    const int64_t gy64 = (N + cta_cols - 1) / cta_cols;
     if (gy64 > 65535) { set_error("N too large"); return DTC_ERR_UNSUPPORTED; }
     const int gy = (int)gy64;
-    const int64_t npad = gy64 * warps * colw;
+    const int64_t npad = gy64 * cta_cols;
     if (h->num_split > 0) {
         const int64_t ncnt = h->num_split * gy * 8;   // per (split, column group, consumer warp)
         if (ncnt > h->counters_len) {
@@ -1262,8 +1513,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     // float4 C stores need an aligned C; the LDG path additionally needs B vectors
     const bool cvec = ((uintptr_t)C % 16 == 0) && (ldc % 4 == 0) && (N % 4 == 0);
     const bool bvec = ((uintptr_t)B % 16 == 0) && (ldb % VW == 0) && (N % VW == 0);
-    const bool use_vec = tma ? cvec : (cvec && bvec);
-    const int path = tma ? 2 : (g_force_path == 3 ? 3 : 1);
+    const bool use_vec = (path == 2 || path == 4) ? cvec : (cvec && bvec);
     // direct path: a pass covers pass_ws warp slices, sized so K x (pass columns) of B stays
     // within ~3/4 of L2 (DTC_PASS_WS overrides: a large value = one unit-major pass)
     const int nws = (int)need;
@@ -1296,7 +1546,7 @@ extern "C" int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, f
 extern "C" int dtc_spmm_launches_per_call(void) { return 1; }
 
 extern "C" int dtc_set_spmm_path(int path) {
-    if (path < 0 || path > 3) { set_error("unknown spmm path %d", path); return DTC_ERR_INVALID; }
+    if (path < 0 || path > 4) { set_error("unknown spmm path %d", path); return DTC_ERR_INVALID; }
     const int prev = g_force_path < 0 ? 0 : g_force_path;
     g_force_path = path == 0 ? DTC_DEFAULT_PATH : path;
     return prev;

@@ -1,4 +1,4 @@
-"""Every dtc_spmm kernel variant (dtc_set_spmm_path: ldg / tma / dir) against oracle O1.
+"""Every dtc_spmm kernel variant (dtc_set_spmm_path: ldg / tma / dir / pad) against oracle O1.
 
 The library default is covered by test_gpu_spmm.py at every config; this module runs the
 same parity bar (tolerance of BASELINE.json north_star, bit-exact for the exact-arithmetic
@@ -16,7 +16,7 @@ from gpu_util import build, dev, spmm, check_tol
 
 pytestmark = pytest.mark.gpu
 
-PATHS = ["ldg", "tma", "dir"]
+PATHS = ["ldg", "tma", "dir", "pad"]
 
 
 @pytest.fixture(params=PATHS)
