@@ -1074,18 +1074,25 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 
 // ============================================================ TMA path with padded rows (path 4)
 // B rows arrive by TMA tile::gather4 in boxes of one 512-byte column slice plus 16 bytes of
-// padding (128 fp32 / 256 fp16 columns + 4 / 8 extra), so consecutive rows of a stage sit
-// 528 bytes apart: 528 = 16 (mod 128) shifts each row by one 16-byte bank group and the
-// fragment reads (lane (g,t): rows 2t and 2t+1, 16-byte chunk g of a 128-byte segment) hit 8
-// distinct bank groups per 8-lane phase -- conflict-free without a swizzle, and 4x fewer TMA
-// ops per byte than 128-byte swizzled boxes (the r01 gather4 ablation was op-rate bound).
-// The gather moves no data through the LSU pipe (the register gather's limiter, ncu
-// l1tex data-pipe 85%); one producer warp runs up to kPadStages blocks ahead.
-// Consumer warps: 2 per slice, each owning 2 x 128-byte segments (64 fp32 / 128 fp16 columns),
-// A fragments built in registers from the occupancy mask one block ahead (as k_spmm_dir).
+// padding (128 fp32 / 256 fp16 columns + 4 / 8 extra), so the 4 rows of one gather4 sit 528
+// bytes apart: 528 = 16 (mod 128) shifts each row by one 16-byte bank group.  One op gathers
+// the block's even rows (SparseAtoB[0,2,4,6]) at slice offset 0, a second the odd rows at
+// offset 2176 (TMA destinations are 128-byte aligned); lane (g,t) reads even row t and odd row
+// t -- its mma rows k=t / k=t+4 (TF32, k permutation as k_spmm_dir) or k=2t / 2t+1 (FP16) --
+// at 16-byte chunk c(g) = (g>>1) + 4(g&1) of a 128-byte segment, so the 8 lanes of an LDS.128
+// phase hit 8 distinct bank groups: conflict-free without a swizzle, and 4x fewer TMA ops per
+// byte than 128-byte swizzled boxes (the r01 gather4 ablation was op-rate bound).  The gather
+// moves no data through the LSU pipe (the register gather's limiter: ncu l1tex data-pipe 85%);
+// one producer warp runs up to pad_stages blocks ahead.  Consumer warps: 2 per slice, each
+// owning 2 x 128-byte segments (64 fp32 / 128 fp16 columns); A fragments are built in
+// registers from the occupancy mask one block ahead (as k_spmm_dir).
+// Column ownership (virtual mma column v <-> chunk c(v)): TF32 thread holds columns
+// seg + 4t + [0,4) and seg + 16 + 4t + [0,4); FP16 seg + 8t + [0,8) and seg + 32 + 8t + [0,8).
 constexpr int kPadBoxElts = 132;                 // 4-byte elements per box row (128 + 4 pad)
 constexpr int kPadRowBytes = kPadBoxElts * 4;    // 528
-constexpr int kPadSliceBytes = 8 * kPadRowBytes; // one TC block x one slice
+constexpr int kPadOddOff = 2176;                 // 17 x 128 >= 4 x 528
+constexpr int kPadSliceBytes = 4352;             // 34 x 128 >= kPadOddOff + 4 x 528
+constexpr int kPadTxBytes = 8 * kPadRowBytes;    // bytes TMA writes per slice per block
 template <int SL>
 constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
@@ -1115,7 +1122,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int CW = 2;                      // 128-byte segments per consumer warp
-    constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;
+    constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
     constexpr int STAGE = SL * kPadSliceBytes;
     constexpr int SLICE_COLS = 4 * COLW1;      // 128 fp32 / 256 fp16 columns per slice
@@ -1141,13 +1148,20 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
 
     if (warp == 2 * SL) {
         // ================= producer: gather4 of 4 B rows x one slice per op =================
-        const uint32_t tx = (uint32_t)nsl * kPadSliceBytes;
-        const int half = lane & 1, jl = lane >> 1;     // lane holds rows 4*half.. of block i0 + jl
+        const uint32_t tx = (uint32_t)nsl * kPadTxBytes;
+        const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
         const int32_t tcol = (int32_t)(col0 * (int64_t)sizeof(typename Tr::elt) / 4);   // 4-byte TMA columns
         auto ids_of = [&](int i0) -> int4 {
             const int i = i0 + jl;
-            return i < nblocks ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(u.bb + i) * 8) + half)
-                               : make_int4(-1, -1, -1, -1);
+            const int4 mine = i < nblocks ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(u.bb + i) * 8) + half)
+                                          : make_int4(-1, -1, -1, -1);
+            int4 o;   // partner's half
+            o.x = __shfl_xor_sync(0xffffffffu, mine.x, 1);
+            o.y = __shfl_xor_sync(0xffffffffu, mine.y, 1);
+            o.z = __shfl_xor_sync(0xffffffffu, mine.z, 1);
+            o.w = __shfl_xor_sync(0xffffffffu, mine.w, 1);
+            return half == 0 ? make_int4(mine.x, mine.z, o.x, o.z)     // rows 0, 2, 4, 6
+                             : make_int4(o.y, o.w, mine.y, mine.w);    // rows 1, 3, 5, 7
         };
         int4 cur = ids_of(0);
         for (int i0 = 0; i0 < nblocks; i0 += 16) {
@@ -1160,7 +1174,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 __syncwarp();
                 if (jl == j) {
                     for (int sl = 0; sl < nsl; ++sl) {
-                        const uint32_t dst = smem_u32(ring + s * STAGE + sl * kPadSliceBytes + half * 4 * kPadRowBytes);
+                        const uint32_t dst = smem_u32(ring + s * STAGE + sl * kPadSliceBytes + half * kPadOddOff);
                         asm volatile(
                             "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                             " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
@@ -1181,15 +1195,16 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int g = lane >> 2, t = lane & 3;
     const int sl = warp >> 1;                            // slice of this warp
     const int64_t n0 = col0 + (int64_t)warp * CW * COLW1;
-    const int64_t base = n0 + 2 * NJ1 * t;
-    const int hoff = NJ1;
+    const int64_t base = n0 + (DT == DTC_TF32 ? 4 : 8) * t;
+    const int hoff = DT == DTC_TF32 ? 16 : 32;
     const bool split = u.split_id >= 0;
     const int pos = 8 * (g & 3) + 2 * t;
     const uint32_t below = (1u << pos) - 1u;
     const bool upper = g >= 4;
-    // smem byte offsets of the thread's rows 2t / 2t+1 at 16-byte chunk g of the warp's first segment
-    const int roff0 = sl * kPadSliceBytes + (2 * t) * kPadRowBytes + (warp & 1) * CW * 128 + g * 16;
-    const int roff1 = roff0 + kPadRowBytes;
+    // smem byte offsets of the thread's even row t / odd row t at chunk c(g) of the warp's first segment
+    const int cg = (g >> 1) + 4 * (g & 1);
+    const int roff0 = sl * kPadSliceBytes + t * kPadRowBytes + (warp & 1) * CW * 128 + cg * 16;
+    const int roff1 = roff0 + kPadOddOff;
 
     float acc[NJ][4];
 #pragma unroll
