@@ -636,7 +636,8 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         TRY(dalloc(&h->atob, 8 * T, s));
         {
             uint8_t* vb = nullptr;
-            TRY(dalloc(&vb, (size_t)std::max<int64_t>(nnz, 1) * elt_size(h->dtype), s));
+            // +16 bytes: the SpMM TMA path bulk-copies 16-byte aligned supersets of value ranges
+            TRY(dalloc(&vb, (size_t)std::max<int64_t>(nnz, 1) * elt_size(h->dtype) + 16, s));
             h->vals = vb;
         }
         k_to_i32<<<grid_for(W + 1, 256, 4096), 256, 0, s>>>(t.nb, h->rwo, W + 1);

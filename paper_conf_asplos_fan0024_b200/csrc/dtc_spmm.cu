@@ -1098,11 +1098,17 @@ constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
     return DTC_PAD_STAGES;
 #else
-    return SL == 1 ? 12 : (SL == 2 ? 6 : 3);
+    return SL == 1 ? 4 : (SL == 2 ? 4 : 3);
 #endif
 }
+// A side of the TMA path: per batch of kPadBatch TC blocks, one bulk copy of the (16-byte
+// aligned superset of the) batch's TCValues -- contiguous, TCOffset[b0] .. TCOffset[b0+16] --
+// and one of its 16 occupancy masks, double buffered.
+constexpr int kPadBatch = 16;
+constexpr int kPadAValBytes = 8320;               // >= 16 blocks x 128 values x 4 B + 16, 128-aligned
+constexpr int kPadASlot = kPadAValBytes + 256;    // + 16 masks
 template <int SL>
-constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * kPadSliceBytes + 128; }
+constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * kPadSliceBytes + 2 * kPadASlot + 128; }
 template <int DT, int SL>
 constexpr int pad_maxregs() {
 #ifdef DTC_PAD_MAXREGS
@@ -1110,6 +1116,24 @@ constexpr int pad_maxregs() {
 #else
     return DT == DTC_FP16 ? 128 : 104;
 #endif
+}
+
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds32_pred(uint32_t a, bool p) {
+    uint32_t v;
+    asm volatile("{\n.reg .pred q;\nsetp.ne.b32 q, %2, 0;\nmov.b32 %0, 0;\n@q ld.shared.u32 %0, [%1];\n}\n"
+                 : "=r"(v) : "r"(a), "r"((int)p));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
+    unsigned short v;
+    asm volatile("{\n.reg .pred q;\nsetp.ne.b32 q, %2, 0;\nmov.b16 %0, 0;\n@q ld.shared.u16 %0, [%1];\n}\n"
+                 : "=h"(v) : "r"(a), "r"((int)p));
+    return (uint32_t)v;
 }
 
 template <int DT, int SL, bool VEC>
@@ -1121,14 +1145,17 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const int32_t* __restrict__ rowmap) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
+    constexpr int ELT = (int)sizeof(typename Tr::elt);
     constexpr int CW = 2;                      // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
     constexpr int STAGE = SL * kPadSliceBytes;
     constexpr int SLICE_COLS = 4 * COLW1;      // 128 fp32 / 256 fp16 columns per slice
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t* ring = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 127) & ~uintptr_t(127));
-    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R];
+    const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
+    const uint32_t aring = ring + R * STAGE;                          // [2][kPadASlot] A batches
+    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[2], bar_aempty[2];
+    __shared__ int s_abyte[2];   // byte offset of the batch's first value inside its A slot
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const Unit u = units[blockIdx.x];
@@ -1142,16 +1169,22 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             mbar_init(&bar_full[i], 1);
             mbar_init(&bar_empty[i], ncons);
         }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&bar_afull[i], 1);
+            mbar_init(&bar_aempty[i], ncons);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
 
     if (warp == 2 * SL) {
-        // ================= producer: gather4 of 4 B rows x one slice per op =================
+        // ================= producer: A batches (bulk copies) + B gather4 (4 rows x one slice per op)
         const uint32_t tx = (uint32_t)nsl * kPadTxBytes;
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
-        const int32_t tcol = (int32_t)(col0 * (int64_t)sizeof(typename Tr::elt) / 4);   // 4-byte TMA columns
-        auto ids_of = [&](int i0) -> int4 {
+        const int32_t tcol = (int32_t)(col0 * ELT / 4);  // 4-byte TMA columns
+        struct BatchMeta { int4 ids; int e0, e1; };
+        auto meta_of = [&](int i0) -> BatchMeta {
+            BatchMeta bm;
             const int i = i0 + jl;
             const int4 mine = i < nblocks ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(u.bb + i) * 8) + half)
                                           : make_int4(-1, -1, -1, -1);
@@ -1160,13 +1193,35 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             o.y = __shfl_xor_sync(0xffffffffu, mine.y, 1);
             o.z = __shfl_xor_sync(0xffffffffu, mine.z, 1);
             o.w = __shfl_xor_sync(0xffffffffu, mine.w, 1);
-            return half == 0 ? make_int4(mine.x, mine.z, o.x, o.z)     // rows 0, 2, 4, 6
-                             : make_int4(o.y, o.w, mine.y, mine.w);    // rows 1, 3, 5, 7
+            bm.ids = half == 0 ? make_int4(mine.x, mine.z, o.x, o.z)     // rows 0, 2, 4, 6
+                               : make_int4(o.y, o.w, mine.y, mine.w);    // rows 1, 3, 5, 7
+            bm.e0 = bm.e1 = 0;
+            if (lane == 0 && i0 < nblocks) {
+                bm.e0 = __ldg(tco + u.bb + i0);
+                bm.e1 = __ldg(tco + u.bb + min(i0 + kPadBatch, nblocks));
+            }
+            return bm;
         };
-        int4 cur = ids_of(0);
-        for (int i0 = 0; i0 < nblocks; i0 += 16) {
-            const int4 nxt = (i0 + 16 < nblocks) ? ids_of(i0 + 16) : make_int4(-1, -1, -1, -1);
-            const int nj = min(16, nblocks - i0);
+        BatchMeta cur = meta_of(0);
+        for (int i0 = 0; i0 < nblocks; i0 += kPadBatch) {
+            const int c = i0 / kPadBatch, aslot = c & 1;
+            const BatchMeta nxt = (i0 + kPadBatch < nblocks) ? meta_of(i0 + kPadBatch) : BatchMeta{make_int4(-1, -1, -1, -1), 0, 0};
+            const int nj = min(kPadBatch, nblocks - i0);
+            if (c >= 2) mbar_wait(&bar_aempty[aslot], ((c >> 1) - 1) & 1);
+            if (lane == 0) {
+                const int64_t lo = ((int64_t)cur.e0 * ELT) & ~int64_t(15);
+                const int64_t hi = ((int64_t)cur.e1 * ELT + 15) & ~int64_t(15);
+                const uint32_t vbytes = (uint32_t)(hi - lo), mbytes = (uint32_t)nj * 16;
+                const uint32_t dst = aring + aslot * kPadASlot;
+                s_abyte[aslot] = (int)((int64_t)cur.e0 * ELT - lo);
+                mbar_arrive_tx(&bar_afull[aslot], vbytes + mbytes);
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(dst), "l"(reinterpret_cast<const uint8_t*>(avals) + lo), "r"(vbytes),
+                             "r"(smem_u32(&bar_afull[aslot])) : "memory");
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(dst + kPadAValBytes), "l"(mask + u.bb + i0), "r"(mbytes),
+                             "r"(smem_u32(&bar_afull[aslot])) : "memory");
+            }
             for (int j = 0; j < nj; ++j) {
                 const int i = i0 + j, s = i % R;
                 if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
@@ -1174,12 +1229,12 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 __syncwarp();
                 if (jl == j) {
                     for (int sl = 0; sl < nsl; ++sl) {
-                        const uint32_t dst = smem_u32(ring + s * STAGE + sl * kPadSliceBytes + half * kPadOddOff);
+                        const uint32_t dst = ring + s * STAGE + sl * kPadSliceBytes + half * kPadOddOff;
                         asm volatile(
                             "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                             " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-                            "l"(&bmap), "r"(tcol + sl * 128), "r"(cur.x), "r"(cur.y), "r"(cur.z), "r"(cur.w),
-                            "r"(smem_u32(&bar_full[s]))
+                            "l"(&bmap), "r"(tcol + sl * 128), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
+                            "r"(cur.ids.w), "r"(smem_u32(&bar_full[s]))
                             : "memory");
                     }
                 }
@@ -1203,8 +1258,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const bool upper = g >= 4;
     // smem byte offsets of the thread's even row t / odd row t at chunk c(g) of the warp's first segment
     const int cg = (g >> 1) + 4 * (g & 1);
-    const int roff0 = sl * kPadSliceBytes + t * kPadRowBytes + (warp & 1) * CW * 128 + cg * 16;
-    const int roff1 = roff0 + kPadOddOff;
+    const uint32_t roff0 = sl * kPadSliceBytes + t * kPadRowBytes + (warp & 1) * CW * 128 + cg * 16;
+    const uint32_t roff1 = roff0 + kPadOddOff;
 
     float acc[NJ][4];
 #pragma unroll
@@ -1218,28 +1273,42 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
     }
-    DirMeta<DT> mt;
-    uint32_t af[FW];
-    if (nblocks > 0) {
-        mt = dir_load_meta<DT>(u.bb, t, atob, mask, tco);
-        dir_load_a<DT>(mt, af, pos, below, upper, avals);
-        if (nblocks > 1) mt = dir_load_meta<DT>(u.bb + 1, t, atob, mask, tco);
-    }
+    uint32_t vaddr = 0, maddr = 0;   // A batch: next block's first value (bytes), mask array
     for (int i = 0; i < nblocks; ++i) {
-        const int s = i % R;
-        uint32_t a[FW];
-#pragma unroll
-        for (int k = 0; k < FW; ++k) a[k] = af[k];
-        if (i + 1 < nblocks) {
-            dir_load_a<DT>(mt, af, pos, below, upper, avals);
-            if (i + 2 < nblocks) mt = dir_load_meta<DT>(u.bb + i + 2, t, atob, mask, tco);
+        const int j = i % kPadBatch, c = i / kPadBatch;
+        if (j == 0) {
+            mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
+            const uint32_t slot = aring + (c & 1) * kPadASlot;
+            vaddr = slot + s_abyte[c & 1];
+            maddr = slot + kPadAValBytes;
         }
+        // S1: A fragment from the occupancy mask and the batch's values (ascending local id, C5)
+        const uint4 m = lds128(maddr + j * 16);
+        const uint32_t wl = upper ? m.y : m.x, wh = upper ? m.w : m.z;
+        const int c0 = __popc(m.x), c01 = c0 + __popc(m.y);
+        const int rl = (upper ? c0 : 0) + __popc(wl & below);
+        const int rh = c01 + (upper ? __popc(m.z) : 0) + __popc(wh & below);
+        const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
+        const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
+        uint32_t a[FW];
+        if constexpr (DT == DTC_TF32) {
+            a[0] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rl, p00)));
+            a[1] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rh, p10)));
+            a[2] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rl + p00), p01)));
+            a[3] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rh + p10), p11)));
+        } else {
+            a[0] = lds16_pred(vaddr + 2 * rl, p00) | (lds16_pred(vaddr + 2 * (rl + p00), p01) << 16);
+            a[1] = lds16_pred(vaddr + 2 * rh, p10) | (lds16_pred(vaddr + 2 * (rh + p10), p11) << 16);
+        }
+        vaddr += ELT * (c01 + __popc(m.z) + __popc(m.w));
+        // S2/S3: B fragments from the padded stage, mma
+        const int s = i % R;
         mbar_wait(&bar_full[s], (i / R) & 1);
-        const uint8_t* st = ring + s * STAGE;
+        const uint32_t st = ring + s * STAGE;
 #pragma unroll
         for (int cw = 0; cw < CW; ++cw) {
-            const uint4 x0 = *reinterpret_cast<const uint4*>(st + roff0 + cw * 128);
-            const uint4 x1 = *reinterpret_cast<const uint4*>(st + roff1 + cw * 128);
+            const uint4 x0 = lds128(st + roff0 + cw * 128);
+            const uint4 x1 = lds128(st + roff1 + cw * 128);
             const uint32_t y0[4] = {x0.x, x0.y, x0.z, x0.w};
             const uint32_t y1[4] = {x1.x, x1.y, x1.z, x1.w};
             if constexpr (DT == DTC_TF32) {
@@ -1256,7 +1325,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             }
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(&bar_empty[s]);
+        if (lane == 0) {
+            mbar_arrive(&bar_empty[s]);
+            if (j == kPadBatch - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[c & 1]);
+        }
         if (u.bb + i + 1 == next_end) {
             store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
 #pragma unroll
