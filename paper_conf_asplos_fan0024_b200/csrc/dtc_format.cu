@@ -491,12 +491,12 @@ struct BuildTemps {
     }
 };
 
-// F4 unit size: ~2.5 windows' worth of TC blocks (measured sweep, DESIGN.md §5:
-// arxiv-like 32, banded 48-64, products-like 128-192, reddit-like 256), clamped to
-// [32, 256] and small enough that there are at least 2 units per SM.
+// F4 unit size: ~2 windows' worth of TC blocks, clamped to [64, 256] (measured sweep for the
+// TMA path, profiles/r01_design_evidence.md: arxiv-like 64, banded 64-128, products-like 128,
+// reddit-like >= 256), and small enough that there are at least 2 units per SM.
 static int auto_unit_blocks(int64_t T, int64_t W) {
-    int64_t target = W > 0 ? (5 * T) / (2 * W) : 32;
-    if (target < 32) target = 32;
+    int64_t target = W > 0 ? (2 * T) / W : 64;
+    if (target < 64) target = 64;
     if (target > 256) target = 256;
     const int64_t cap = T / (2 * (int64_t)num_sms());
     if (target > cap) target = cap < 8 ? 8 : cap;

@@ -1529,7 +1529,7 @@ static int64_t l2_bytes() {
 
 static int g_force_path = -1;   // 1 = register gather via smem A chunks, 2 = TMA gather4, 3 = direct (DTC_SPMM_PATH=ldg|tma|dir)
 #ifndef DTC_DEFAULT_PATH
-#define DTC_DEFAULT_PATH 1
+#define DTC_DEFAULT_PATH 4   // TMA padded-row path (falls back to path 1 where TMA cannot describe B)
 #endif
 static int env_path() {
     const char* e = getenv("DTC_SPMM_PATH");
