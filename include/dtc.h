@@ -150,6 +150,14 @@ int dtc_spmm_launches_per_call(void);
  * (0 if it was the default), or DTC_ERR_INVALID for an unknown path. */
 int dtc_set_spmm_path(int path);
 
+/* Diagnostics (the paper's per-SM busy/idle methodology, Fig. 3 P:152-160 / Fig. 15):
+ * while enabled, each CTA of the TMA-path kernel writes 8 int64 to dev_buf[cta*8 ..]:
+ * {cta, smid, t_start, t_first_issue, t_first_data, t_consumer_done, num_tc_blocks,
+ * t_producer_done}, times in ns of the %globaltimer.  dev_buf is a caller-owned device buffer of
+ * capacity_ctas*8 int64; launches with more CTAs than capacity_ctas are not traced.
+ * capacity_ctas = 0 disables.  Process-wide.  Errors: INVALID. */
+int dtc_set_trace(void* dev_buf, int64_t capacity_ctas);
+
 void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory */
 
 /* ------------------------------------------------------------ reordering (NEXT-1)

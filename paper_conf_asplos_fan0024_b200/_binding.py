@@ -76,6 +76,7 @@ def lib():
             L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_launches_per_call.argtypes = []
             L.dtc_set_spmm_path.argtypes = [ctypes.c_int]
+            L.dtc_set_trace.argtypes = [_vp, _i64]
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
@@ -124,6 +125,17 @@ def launches_per_call() -> int:
 
 
 SPMM_PATHS = {"default": 0, "ldg": 1, "tma": 2, "dir": 3, "pad": 4}
+
+
+def set_trace(buf=None) -> None:
+    """Enable (CUDA int64 tensor of shape [ctas, 8]) or disable (None) the per-CTA timeline."""
+    if buf is None:
+        _check(lib().dtc_set_trace(None, 0), "dtc_set_trace")
+        return
+    import torch
+    if buf.dtype != torch.int64 or not buf.is_cuda or buf.dim() != 2 or buf.shape[1] != 8:
+        raise TypeError("trace buffer must be a CUDA int64 tensor [ctas, 8]")
+    _check(lib().dtc_set_trace(ctypes.c_void_p(buf.data_ptr()), buf.shape[0]), "dtc_set_trace")
 
 
 def set_spmm_path(path) -> int:

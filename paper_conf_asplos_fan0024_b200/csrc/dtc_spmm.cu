@@ -1118,6 +1118,16 @@ constexpr int pad_maxregs() {
 #endif
 }
 
+__device__ __forceinline__ int64_t gtimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return (int64_t)t;
+}
+__device__ __forceinline__ int smid() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return (int)r;
+}
 __device__ __forceinline__ uint4 lds128(uint32_t a) {
     uint4 v;
     asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
@@ -1142,10 +1152,18 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
-           const int32_t* __restrict__ rowmap) {
+           const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
+    // optional per-CTA timeline (dtc_set_trace): {cta, smid, t_start, t_first_issue, t_first_data,
+    // t_consumer_done, nblocks, t_producer_done} in %globaltimer ns
+    int64_t* tr = trace ? trace + ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * 8 : nullptr;
+    if (tr && threadIdx.x == 0) {
+        tr[0] = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
+        tr[1] = smid();
+        tr[2] = gtimer();
+    }
     constexpr int CW = 2;                      // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
@@ -1227,6 +1245,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
                 if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
                 __syncwarp();
+                if (tr && i == 0 && lane == 0) tr[3] = gtimer();
                 if (jl == j) {
                     for (int sl = 0; sl < nsl; ++sl) {
                         const uint32_t dst = ring + s * STAGE + sl * kPadSliceBytes + half * kPadOddOff;
@@ -1241,6 +1260,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 __syncwarp();
             }
             cur = nxt;
+        }
+        if (tr && lane == 0) {
+            tr[6] = nblocks;
+            tr[7] = gtimer();
         }
         return;
     }
@@ -1304,6 +1327,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         // S2/S3: B fragments from the padded stage, mma
         const int s = i % R;
         mbar_wait(&bar_full[s], (i / R) & 1);
+        if (tr && i == 0 && threadIdx.x == 0) tr[4] = gtimer();
         const uint32_t st = ring + s * STAGE;
 #pragma unroll
         for (int cw = 0; cw < CW; ++cw) {
@@ -1343,10 +1367,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     }
     if (!split) {
         while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
-        return;
+    } else {
+        int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
+        split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
     }
-    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+    if (tr && threadIdx.x == 0) tr[5] = gtimer();
 }
 
 // ============================================================ host side
@@ -1398,6 +1423,10 @@ static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
+
+// optional per-CTA timeline of the TMA path (dtc_set_trace; diagnostics, profiles/)
+static int64_t* g_trace = nullptr;
+static int64_t g_trace_cap = 0;
 
 struct LaunchArgs {
     dtc_format* h;
@@ -1473,7 +1502,8 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
     k_spmm_pad<DT, SL, VEC><<<grid, (2 * SL + 1) * 32, smem, a.s>>>(
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
-        a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap);
+        a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
+        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr);
     return cudaGetLastError();
 }
 
@@ -1631,6 +1661,13 @@ extern "C" int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, f
 }
 
 extern "C" int dtc_spmm_launches_per_call(void) { return 1; }
+
+extern "C" int dtc_set_trace(void* dev_buf, int64_t capacity_ctas) {
+    if (capacity_ctas < 0 || (capacity_ctas > 0 && !dev_buf)) { set_error("bad trace buffer"); return DTC_ERR_INVALID; }
+    g_trace = capacity_ctas ? reinterpret_cast<int64_t*>(dev_buf) : nullptr;
+    g_trace_cap = capacity_ctas;
+    return DTC_OK;
+}
 
 extern "C" int dtc_set_spmm_path(int path) {
     if (path < 0 || path > 4) { set_error("unknown spmm path %d", path); return DTC_ERR_INVALID; }
