@@ -1088,11 +1088,17 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 // registers from the occupancy mask one block ahead (as k_spmm_dir).
 // Column ownership (virtual mma column v <-> chunk c(v)): TF32 thread holds columns
 // seg + 4t + [0,4) and seg + 16 + 4t + [0,4); FP16 seg + 8t + [0,8) and seg + 32 + 8t + [0,8).
-constexpr int kPadBoxElts = 132;                 // 4-byte elements per box row (128 + 4 pad)
-constexpr int kPadRowBytes = kPadBoxElts * 4;    // 528
-constexpr int kPadOddOff = 2176;                 // 17 x 128 >= 4 x 528
-constexpr int kPadSliceBytes = 4352;             // 34 x 128 >= kPadOddOff + 4 x 528
-constexpr int kPadTxBytes = 8 * kPadRowBytes;    // bytes TMA writes per slice per block
+// Slice geometry, SEG = 128-byte segments per slice row: 4 (512-byte slices, 4-byte TMA
+// elements, box 132) or 8 (1 KB slices, 8-byte TMA elements, box 130 -- one gather4 op moves
+// 2x the bytes, for B rows of >= 1 KB).  Row pitch SEG*128 + 16 (= 16 mod 128).
+template <int SEG> constexpr int pad_row_bytes() { return SEG * 128 + 16; }
+template <int SEG> constexpr int pad_box_elts() { return SEG == 4 ? 132 : 130; }
+template <int SEG> constexpr int pad_tma_elt() { return SEG == 4 ? 4 : 8; }
+template <int SEG> constexpr int pad_odd_off() { return (4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
+template <int SEG> constexpr int pad_slice_bytes() { return (pad_odd_off<SEG>() + 4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
+template <int SEG> constexpr int pad_tx_bytes() { return 8 * pad_row_bytes<SEG>(); }
+static_assert(pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16, "row pitch must be 16 mod 128");
+static_assert(pad_box_elts<4>() * 4 == pad_row_bytes<4>() && pad_box_elts<8>() * 8 == pad_row_bytes<8>(), "box");
 template <int SL>
 constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
@@ -1107,8 +1113,8 @@ constexpr int pad_stages() {
 constexpr int kPadBatch = 16;
 constexpr int kPadAValBytes = 8320;               // >= 16 blocks x 128 values x 4 B + 16, 128-aligned
 constexpr int kPadASlot = kPadAValBytes + 256;    // + 16 masks
-template <int SL>
-constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * kPadSliceBytes + 2 * kPadASlot + 128; }
+template <int SL, int SEG>
+constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * kPadASlot + 128; }
 template <int DT, int SL>
 constexpr int pad_maxregs() {
 #ifdef DTC_PAD_MAXREGS
@@ -1146,8 +1152,8 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
     return (uint32_t)v;
 }
 
-template <int DT, int SL, bool VEC>
-__global__ void __launch_bounds__((2 * SL + 1) * 32, 65536 / ((2 * SL + 1) * 32 * pad_maxregs<DT, SL>()))
+template <int DT, int SL, int SEG, bool VEC>
+__global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
@@ -1167,8 +1173,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     constexpr int CW = 2;                      // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
-    constexpr int STAGE = SL * kPadSliceBytes;
-    constexpr int SLICE_COLS = 4 * COLW1;      // 128 fp32 / 256 fp16 columns per slice
+    constexpr int WPS = SEG / 2;               // consumer warps per slice
+    constexpr int ROWB = pad_row_bytes<SEG>(), ODD = pad_odd_off<SEG>(), SLB = pad_slice_bytes<SEG>();
+    constexpr int STAGE = SL * SLB;
+    constexpr int SLICE_COLS = SEG * COLW1;    // 128 / 256 fp32 or 256 / 512 fp16 columns per slice
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
     const uint32_t aring = ring + R * STAGE;                          // [2][kPadASlot] A batches
@@ -1180,7 +1188,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int64_t col0 = (int64_t)blockIdx.y * SL * SLICE_COLS;          // first C column of the CTA
     const int64_t nsl64 = (N - col0 + SLICE_COLS - 1) / SLICE_COLS;
     const int nsl = nsl64 < SL ? (int)nsl64 : SL;
-    const int ncons = 2 * nsl;
+    const int ncons = WPS * nsl;
     const int nblocks = u.be - u.bb;
     if (threadIdx.x == 0) {
         for (int i = 0; i < R; ++i) {
@@ -1195,11 +1203,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     }
     __syncthreads();
 
-    if (warp == 2 * SL) {
+    if (warp == WPS * SL) {
         // ================= producer: A batches (bulk copies) + B gather4 (4 rows x one slice per op)
-        const uint32_t tx = (uint32_t)nsl * kPadTxBytes;
+        const uint32_t tx = (uint32_t)nsl * pad_tx_bytes<SEG>();
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
-        const int32_t tcol = (int32_t)(col0 * ELT / 4);  // 4-byte TMA columns
+        const int32_t tcol = (int32_t)(col0 * ELT / pad_tma_elt<SEG>());  // TMA columns (4- or 8-byte elements)
         struct BatchMeta { int4 ids; int e0, e1; };
         auto meta_of = [&](int i0) -> BatchMeta {
             BatchMeta bm;
@@ -1248,7 +1256,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 if (tr && i == 0 && lane == 0) tr[3] = gtimer();
                 if (jl == j) {
                     for (int sl = 0; sl < nsl; ++sl) {
-                        const uint32_t dst = ring + s * STAGE + sl * kPadSliceBytes + half * kPadOddOff;
+                        const uint32_t dst = ring + s * STAGE + sl * SLB + half * ODD;
                         asm volatile(
                             "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                             " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
@@ -1271,7 +1279,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
 
     // ================= consumers (S1 A fragments, S3 mma, S4/S5) =================
     const int g = lane >> 2, t = lane & 3;
-    const int sl = warp >> 1;                            // slice of this warp
+    const int sl = warp / WPS;                           // slice of this warp
     const int64_t n0 = col0 + (int64_t)warp * CW * COLW1;
     const int64_t base = n0 + (DT == DTC_TF32 ? 4 : 8) * t;
     const int hoff = DT == DTC_TF32 ? 16 : 32;
@@ -1281,8 +1289,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const bool upper = g >= 4;
     // smem byte offsets of the thread's even row t / odd row t at chunk c(g) of the warp's first segment
     const int cg = (g >> 1) + 4 * (g & 1);
-    const uint32_t roff0 = sl * kPadSliceBytes + t * kPadRowBytes + (warp & 1) * CW * 128 + cg * 16;
-    const uint32_t roff1 = roff0 + kPadOddOff;
+    const uint32_t roff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + cg * 16;
+    const uint32_t roff1 = roff0 + ODD;
 
     float acc[NJ][4];
 #pragma unroll
@@ -1410,17 +1418,18 @@ static bool make_bmap(CUtensorMap* map, const void* B, int64_t K, int64_t N, int
 
 // Tensor map of B viewed as 4-byte elements (fp16 pairs for FP16): K rows x N*elt/4 columns,
 // gather4 boxes of kPadBoxElts x 1, no swizzle (rows land 528 bytes apart, see k_spmm_pad).
-static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype) {
+static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype, int seg) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return false;
     const int elt = elt_size(dtype);
-    cuuint64_t dims[2] = {(cuuint64_t)(N * elt / 4), (cuuint64_t)K};
+    const int te = seg == 4 ? 4 : 8;   // TMA element bytes
+    cuuint64_t dims[2] = {(cuuint64_t)(N * elt / te), (cuuint64_t)K};
     cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
-    cuuint32_t box[2] = {(cuuint32_t)kPadBoxElts, 1};
+    cuuint32_t box[2] = {(cuuint32_t)(seg == 4 ? pad_box_elts<4>() : pad_box_elts<8>()), 1};
     cuuint32_t estr[2] = {1, 1};
-    CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(B), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    CUresult r = enc(map, te == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2,
+                     const_cast<void*>(B), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
 
@@ -1438,6 +1447,7 @@ struct LaunchArgs {
     int64_t npad;
     cudaStream_t s;
     int nws, pass_ws;   // direct path: warp slices of N, slices per L2-resident pass
+    int seg;            // TMA padded path: 128-byte segments per slice (4 or 8)
 };
 
 template <int DT, int WARPS>
@@ -1491,16 +1501,16 @@ static cudaError_t launch_dir(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
-template <int DT, int SL, bool VEC>
+template <int DT, int SL, int SEG, bool VEC>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
-    const size_t smem = pad_smem_bytes<SL>();
+    const size_t smem = pad_smem_bytes<SL, SEG>();
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(k_spmm_pad<DT, SL, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(k_spmm_pad<DT, SL, SEG, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = true;
     }
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
-    k_spmm_pad<DT, SL, VEC><<<grid, (2 * SL + 1) * 32, smem, a.s>>>(
+    k_spmm_pad<DT, SL, SEG, VEC><<<grid, (SL * SEG / 2 + 1) * 32, smem, a.s>>>(
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
         (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr);
@@ -1509,11 +1519,12 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
 
 template <int DT, bool VEC>
 static cudaError_t dispatch(int warps, int path, const LaunchArgs& a, const CUtensorMap& map) {
-    if (path == 4) {
-        switch (warps) {   // warps = slices per CTA here
-            case 1: return launch_pad<DT, 1, VEC>(a, map);
-            case 2: return launch_pad<DT, 2, VEC>(a, map);
-            default: return launch_pad<DT, 4, VEC>(a, map);
+    if (path == 4) {   // warps = slices per CTA, a.seg = segments per slice
+        if (a.seg == 8) return warps >= 2 ? launch_pad<DT, 2, 8, VEC>(a, map) : launch_pad<DT, 1, 8, VEC>(a, map);
+        switch (warps) {
+            case 1: return launch_pad<DT, 1, 4, VEC>(a, map);
+            case 2: return launch_pad<DT, 2, 4, VEC>(a, map);
+            default: return launch_pad<DT, 4, 4, VEC>(a, map);
         }
     }
     const bool tma = path == 2;
@@ -1586,7 +1597,14 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
                         h->K < (int64_t(1) << 31) && N < (int64_t(1) << 31);
     int path = g_force_path == 3 ? 3 : 1;
     if (g_force_path == 2 && tma_ok && make_bmap(&map, B, h->K, N, ldb, h->dtype)) path = 2;
-    if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype)) path = 4;
+    // TMA padded path: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB, else 512 B
+    int seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : 4;
+    {
+        const char* e = getenv("DTC_PAD_SEG");
+        if (e && atoi(e) == 4) seg = 4;
+    }
+    if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg))
+        path = 4;
     // columns per warp: the 128B-swizzled TMA path one 128-byte slice per warp, the others two
     const int colw_tma = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
     const int colw_ldg = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW * ldg_colchunks<DTC_FP16>()
@@ -1596,12 +1614,13 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     int warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
     int64_t cta_cols = (int64_t)warps * colw;
     if (path == 4) {
-        // warps := slices (of 512 bytes of a B row) per CTA; two consumer warps per slice
-        const int64_t slice_cols = 512 / elt;
+        // warps := slices (of seg x 128 bytes of a B row) per CTA; seg/2 consumer warps per slice,
+        // at most 4 consumer warps per CTA by default (DTC_PAD_SL overrides the slice cap)
+        const int64_t slice_cols = seg * 128 / elt;
         const int64_t nsl = (N + slice_cols - 1) / slice_cols;
         const char* e = getenv("DTC_PAD_SL");
-        const int slmax = (e && atoi(e) > 0) ? atoi(e) : 2;
-        warps = nsl >= 4 && slmax >= 4 ? 4 : (nsl >= 2 && slmax >= 2 ? 2 : 1);
+        const int slmax = (e && atoi(e) > 0) ? atoi(e) : (seg == 8 ? 1 : 2);
+        warps = nsl >= 4 && slmax >= 4 && seg == 4 ? 4 : (nsl >= 2 && slmax >= 2 ? 2 : 1);
         cta_cols = warps * slice_cols;
     }
     const int64_t gy64 = (N + cta_cols - 1) / cta_cols;
@@ -1642,7 +1661,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
         pass_ws = (int)std::min<int64_t>(nws, std::max<int64_t>(1, fit));
         if (e && atoi(e) > 0) pass_ws = std::min(nws, atoi(e));
     }
-    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws};
+    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws, seg};
     cudaError_t e;
     if (h->dtype == DTC_FP16)
         e = use_vec ? dispatch<DTC_FP16, true>(warps, path, a, map) : dispatch<DTC_FP16, false>(warps, path, a, map);
