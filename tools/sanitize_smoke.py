@@ -6,13 +6,15 @@ import numpy as np
 import torch
 import datagen
 from datagen import configs
-from paper_conf_asplos_fan0024_b200 import Format
+from paper_conf_asplos_fan0024_b200 import Format, set_spmm_path
 
 cfg = configs.get("c1")
 rp, ci = configs.make_pattern(cfg)
-for dtype in ("tf32", "fp16"):
+for path in ("default", "ldg", "dir"):
+  set_spmm_path(path)
+  for dtype in ("tf32", "fp16"):
     v = configs.make_values(cfg, len(ci))
-    for N in (32, 37, 128):
+    for N in ((32, 37, 128, 256, 512) if path == "default" else (37, 128)):
         B = datagen.uniform(1, 2, cfg.K * N).reshape(cfg.K, N)
         if dtype == "fp16":
             v, B = v.astype(np.float16), B.astype(np.float16)
