@@ -1619,7 +1619,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
         const int64_t slice_cols = seg * 128 / elt;
         const int64_t nsl = (N + slice_cols - 1) / slice_cols;
         const char* e = getenv("DTC_PAD_SL");
-        const int slmax = (e && atoi(e) > 0) ? atoi(e) : (seg == 8 ? 1 : 2);
+        const int slmax = (e && atoi(e) > 0) ? atoi(e) : 2;
         warps = nsl >= 4 && slmax >= 4 && seg == 4 ? 4 : (nsl >= 2 && slmax >= 2 ? 2 : 1);
         cta_cols = warps * slice_cols;
     }
