@@ -1092,13 +1092,14 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 // elements, box 132) or 8 (1 KB slices, 8-byte TMA elements, box 130 -- one gather4 op moves
 // 2x the bytes, for B rows of >= 1 KB).  Row pitch SEG*128 + 16 (= 16 mod 128).
 template <int SEG> constexpr int pad_row_bytes() { return SEG * 128 + 16; }
-template <int SEG> constexpr int pad_box_elts() { return SEG == 4 ? 132 : 130; }
-template <int SEG> constexpr int pad_tma_elt() { return SEG == 4 ? 4 : 8; }
+template <int SEG> constexpr int pad_box_elts() { return SEG == 2 ? 68 : (SEG == 4 ? 132 : 130); }
+template <int SEG> constexpr int pad_tma_elt() { return SEG == 8 ? 8 : 4; }
 template <int SEG> constexpr int pad_odd_off() { return (4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_slice_bytes() { return (pad_odd_off<SEG>() + 4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_tx_bytes() { return 8 * pad_row_bytes<SEG>(); }
 static_assert(pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16, "row pitch must be 16 mod 128");
-static_assert(pad_box_elts<4>() * 4 == pad_row_bytes<4>() && pad_box_elts<8>() * 8 == pad_row_bytes<8>(), "box");
+static_assert(pad_box_elts<4>() * 4 == pad_row_bytes<4>() && pad_box_elts<8>() * 8 == pad_row_bytes<8>() &&
+                  pad_box_elts<2>() * 4 == pad_row_bytes<2>() && pad_row_bytes<2>() % 128 == 16, "box");
 template <int SL>
 constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
@@ -1112,9 +1113,12 @@ constexpr int pad_stages() {
 // and one of its 16 occupancy masks, double buffered.
 constexpr int kPadBatch = 16;
 constexpr int kPadAValBytes = 8320;               // >= 16 blocks x 128 values x 4 B + 16, 128-aligned
-constexpr int kPadASlot = kPadAValBytes + 256;    // + 16 masks
+constexpr int kPadAIdsOff = kPadAValBytes + 256;  // + 16 masks
+constexpr int kPadASlot = kPadAIdsOff + 512;       // + 16 x 8 SparseAtoB ids (hybrid LDG warps)
 template <int SL, int SEG>
-constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * kPadASlot + 128; }
+constexpr size_t pad_smem_bytes_() { return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * kPadASlot + 128; }
+template <int SL, int SEG>
+constexpr size_t pad_smem_bytes() { return pad_smem_bytes_<SL, SEG>(); }
 template <int DT, int SL>
 constexpr int pad_maxregs() {
 #ifdef DTC_PAD_MAXREGS
@@ -1134,6 +1138,11 @@ __device__ __forceinline__ int smid() {
     asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
     return (int)r;
 }
+__device__ __forceinline__ uint2 lds64(uint32_t a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
 __device__ __forceinline__ uint4 lds128(uint32_t a) {
     uint4 v;
     asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
@@ -1152,13 +1161,15 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
     return (uint32_t)v;
 }
 
-template <int DT, int SL, int SEG, bool VEC>
-__global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL>()))
+template <int DT, int SL, int SEG, int NL, bool VEC>
+__global__ void __launch_bounds__((SL * SEG / 2 + NL + 1) * 32,
+                                  65536 / ((SL * SEG / 2 + NL + 1) * 32 * pad_maxregs<DT, SL>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
-           const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace) {
+           const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
+           int64_t ldb) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1185,10 +1196,15 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const Unit u = units[blockIdx.x];
-    const int64_t col0 = (int64_t)blockIdx.y * SL * SLICE_COLS;          // first C column of the CTA
+    // CTA columns: SL TMA slices, then NL register-gather (LSU) warps of CW segments each (hybrid:
+    // the TMA engine and the LSU pipe gather different columns of the same TC blocks concurrently)
+    constexpr int CTA_COLS = SL * SLICE_COLS + NL * CW * COLW1;
+    constexpr int WT = SL * WPS;               // TMA consumer warps
+    const int64_t col0 = (int64_t)blockIdx.y * CTA_COLS;               // first C column of the CTA
     const int64_t nsl64 = (N - col0 + SLICE_COLS - 1) / SLICE_COLS;
-    const int nsl = nsl64 < SL ? (int)nsl64 : SL;
-    const int ncons = WPS * nsl;
+    const int nsl = nsl64 < SL ? (int)(nsl64 > 0 ? nsl64 : 0) : SL;
+    const int ncons = WPS * nsl;               // B-stage consumers
+    const int nacons = ncons + NL;             // A-batch consumers
     const int nblocks = u.be - u.bb;
     if (threadIdx.x == 0) {
         for (int i = 0; i < R; ++i) {
@@ -1197,13 +1213,13 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&bar_afull[i], 1);
-            mbar_init(&bar_aempty[i], ncons);
+            mbar_init(&bar_aempty[i], nacons);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
 
-    if (warp == WPS * SL) {
+    if (warp == WT + NL) {
         // ================= producer: A batches (bulk copies) + B gather4 (4 rows x one slice per op)
         const uint32_t tx = (uint32_t)nsl * pad_tx_bytes<SEG>();
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
@@ -1238,9 +1254,16 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 const int64_t lo = ((int64_t)cur.e0 * ELT) & ~int64_t(15);
                 const int64_t hi = ((int64_t)cur.e1 * ELT + 15) & ~int64_t(15);
                 const uint32_t vbytes = (uint32_t)(hi - lo), mbytes = (uint32_t)nj * 16;
+                const uint32_t ibytes = NL > 0 ? (uint32_t)nj * 32 : 0u;
                 const uint32_t dst = aring + aslot * kPadASlot;
                 s_abyte[aslot] = (int)((int64_t)cur.e0 * ELT - lo);
-                mbar_arrive_tx(&bar_afull[aslot], vbytes + mbytes);
+                mbar_arrive_tx(&bar_afull[aslot], vbytes + mbytes + ibytes);
+                if (NL > 0)
+                    asm volatile(
+                        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                            dst + kPadAIdsOff),
+                        "l"(atob + (int64_t)(u.bb + i0) * 8), "r"(ibytes), "r"(smem_u32(&bar_afull[aslot]))
+                        : "memory");
                 asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                              ::"r"(dst), "l"(reinterpret_cast<const uint8_t*>(avals) + lo), "r"(vbytes),
                              "r"(smem_u32(&bar_afull[aslot])) : "memory");
@@ -1260,7 +1283,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                         asm volatile(
                             "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                             " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-                            "l"(&bmap), "r"(tcol + sl * 128), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
+                            "l"(&bmap), "r"(tcol + sl * (SEG * 128 / pad_tma_elt<SEG>())), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
                             "r"(cur.ids.w), "r"(smem_u32(&bar_full[s]))
                             : "memory");
                     }
@@ -1272,6 +1295,138 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (tr && lane == 0) {
             tr[6] = nblocks;
             tr[7] = gtimer();
+        }
+        return;
+    }
+    if (NL > 0 && warp >= WT) {
+        // ================= hybrid register-gather warp (S1 from the A batch, S2 on the LSU path)
+        const int g = lane >> 2, t = lane & 3;
+        constexpr int VW = Tr::VW;
+        const int64_t n0 = col0 + SL * SLICE_COLS + (int64_t)(warp - WT) * CW * COLW1;
+        const bool active = n0 < N;
+        const int64_t bcol = n0 + (int64_t)VW * g;
+        const int64_t base = n0 + 2 * NJ1 * t;
+        const int hoff = NJ1;
+        const bool split = u.split_id >= 0;
+        const int pos = 8 * (g & 3) + 2 * t;
+        const uint32_t below = (1u << pos) - 1u;
+        const bool upper = g >= 4;
+        const char* bthr = reinterpret_cast<const char*>(B) + bcol * (int64_t)ELT;
+        const uint64_t ldb_bytes = (uint64_t)ldb * ELT;
+        auto gather = [&](int row, int cw) -> V16 {
+            const bool ok = active && row >= 0 && (bcol + cw * COLW1) < N;
+            const char* p = ok ? bthr + (uint64_t)(uint32_t)row * ldb_bytes + cw * COLW1 * ELT
+                               : reinterpret_cast<const char*>(g_zero_line);
+            const uint4 x = __ldg(reinterpret_cast<const uint4*>(p));
+            V16 v;
+            v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
+            return v;
+        };
+        float acc[NJ][4];
+#pragma unroll
+        for (int jx = 0; jx < NJ; ++jx) acc[jx][0] = acc[jx][1] = acc[jx][2] = acc[jx][3] = 0.f;
+        int cur = u.wb;
+        int next_end = INT_MAX;
+        if (!split) {
+            while (cur < u.we && rwo[cur + 1] <= u.bb) {
+                if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                ++cur;
+            }
+            next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+        }
+        uint32_t vaddr = 0, maddr = 0, iaddr = 0, niaddr = 0;
+        V16 b0[CW], b1[CW];
+        if (nblocks > 0) {
+            mbar_wait(&bar_afull[0], 0);
+            const uint32_t slot = aring;
+            vaddr = slot + s_abyte[0];
+            maddr = slot + kPadAValBytes;
+            iaddr = niaddr = slot + kPadAIdsOff;
+            const uint2 id = lds64(iaddr + 8 * t);
+#pragma unroll
+            for (int cw = 0; cw < CW; ++cw) { b0[cw] = gather((int)id.x, cw); b1[cw] = gather((int)id.y, cw); }
+        }
+        for (int i = 0; i < nblocks; ++i) {
+            const int j = i % kPadBatch, c = i / kPadBatch;
+            // A fragment of block i (batch c)
+            const uint4 m = lds128(maddr + j * 16);
+            const uint32_t wl = upper ? m.y : m.x, wh = upper ? m.w : m.z;
+            const int c0 = __popc(m.x), c01 = c0 + __popc(m.y);
+            const int rl = (upper ? c0 : 0) + __popc(wl & below);
+            const int rh = c01 + (upper ? __popc(m.z) : 0) + __popc(wh & below);
+            const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
+            const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
+            uint32_t a[FW];
+            if constexpr (DT == DTC_TF32) {
+                a[0] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rl, p00)));
+                a[1] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rh, p10)));
+                a[2] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rl + p00), p01)));
+                a[3] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rh + p10), p11)));
+            } else {
+                a[0] = lds16_pred(vaddr + 2 * rl, p00) | (lds16_pred(vaddr + 2 * (rl + p00), p01) << 16);
+                a[1] = lds16_pred(vaddr + 2 * rh, p10) | (lds16_pred(vaddr + 2 * (rh + p10), p11) << 16);
+            }
+            vaddr += ELT * (c01 + __popc(m.z) + __popc(m.w));
+            // B rows of block i+1 (its ids may live in the next batch)
+            V16 n0v[CW], n1v[CW];
+            if (i + 1 < nblocks) {
+                const int jn = (i + 1) % kPadBatch;
+                if (jn == 0) {
+                    const int cn = c + 1;
+                    mbar_wait(&bar_afull[cn & 1], (cn >> 1) & 1);
+                    niaddr = aring + (cn & 1) * kPadASlot + kPadAIdsOff;
+                }
+                const uint2 id = lds64(niaddr + jn * 32 + 8 * t);
+#pragma unroll
+                for (int cw = 0; cw < CW; ++cw) { n0v[cw] = gather((int)id.x, cw); n1v[cw] = gather((int)id.y, cw); }
+            }
+            if (active) {
+                if constexpr (DT == DTC_TF32) {
+                    const uint32_t aa[4] = {a[0], a[1], a[2], a[3]};
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                        for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[cw * NJ1 + jj], aa, b0[cw].w[jj], b1[cw].w[jj]);
+                } else {
+                    const uint32_t aa[2] = {a[0], a[1]};
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw)
+#pragma unroll
+                        for (int jj = 0; jj < NJ1; ++jj) {
+                            const uint32_t bb = __byte_perm(b0[cw].w[jj >> 1], b1[cw].w[jj >> 1], (jj & 1) ? 0x7632 : 0x5410);
+                            mma_f16(acc[cw * NJ1 + jj], aa, bb);
+                        }
+                }
+            }
+#pragma unroll
+            for (int cw = 0; cw < CW; ++cw) { b0[cw] = n0v[cw]; b1[cw] = n1v[cw]; }
+            if (j == kPadBatch - 1 || i == nblocks - 1) {   // done with batch c (values, masks, ids)
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bar_aempty[c & 1]);
+                if (i + 1 < nblocks) {
+                    const uint32_t slot = aring + ((c + 1) & 1) * kPadASlot;
+                    vaddr = slot + s_abyte[(c + 1) & 1];
+                    maddr = slot + kPadAValBytes;
+                }
+            }
+            if (u.bb + i + 1 == next_end) {
+                if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+#pragma unroll
+                for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+                ++cur;
+                while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
+                    if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                    ++cur;
+                }
+                next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+            }
+        }
+        if (!active) return;
+        if (!split) {
+            while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
+        } else {
+            int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
+            split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
         }
         return;
     }
@@ -1422,10 +1577,10 @@ static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N,
     EncodeTiledFn enc = encode_fn();
     if (!enc) return false;
     const int elt = elt_size(dtype);
-    const int te = seg == 4 ? 4 : 8;   // TMA element bytes
+    const int te = seg == 8 ? 8 : 4;   // TMA element bytes
     cuuint64_t dims[2] = {(cuuint64_t)(N * elt / te), (cuuint64_t)K};
     cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
-    cuuint32_t box[2] = {(cuuint32_t)(seg == 4 ? pad_box_elts<4>() : pad_box_elts<8>()), 1};
+    cuuint32_t box[2] = {(cuuint32_t)(seg == 2 ? pad_box_elts<2>() : seg == 4 ? pad_box_elts<4>() : pad_box_elts<8>()), 1};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(map, te == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2,
                      const_cast<void*>(B), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -1447,7 +1602,8 @@ struct LaunchArgs {
     int64_t npad;
     cudaStream_t s;
     int nws, pass_ws;   // direct path: warp slices of N, slices per L2-resident pass
-    int seg;            // TMA padded path: 128-byte segments per slice (4 or 8)
+    int seg;            // TMA padded path: 128-byte segments per slice (2, 4 or 8)
+    int nl;             // TMA padded path: register-gather (LSU) warps per CTA (hybrid), 0 = none
 };
 
 template <int DT, int WARPS>
@@ -1501,30 +1657,35 @@ static cudaError_t launch_dir(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
-template <int DT, int SL, int SEG, bool VEC>
+template <int DT, int SL, int SEG, int NL, bool VEC>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     const size_t smem = pad_smem_bytes<SL, SEG>();
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(k_spmm_pad<DT, SL, SEG, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(k_spmm_pad<DT, SL, SEG, NL, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = true;
     }
     dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
-    k_spmm_pad<DT, SL, SEG, VEC><<<grid, (SL * SEG / 2 + 1) * 32, smem, a.s>>>(
+    k_spmm_pad<DT, SL, SEG, NL, VEC><<<grid, (SL * SEG / 2 + NL + 1) * 32, smem, a.s>>>(
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
-        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr);
+        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb);
     return cudaGetLastError();
 }
 
 template <int DT, bool VEC>
 static cudaError_t dispatch(int warps, int path, const LaunchArgs& a, const CUtensorMap& map) {
-    if (path == 4) {   // warps = slices per CTA, a.seg = segments per slice
-        if (a.seg == 8) return warps >= 2 ? launch_pad<DT, 2, 8, VEC>(a, map) : launch_pad<DT, 1, 8, VEC>(a, map);
+    if (path == 4) {   // warps = TMA slices per CTA, a.seg = segments per slice, a.nl = LSU warps
+        if (a.nl > 0) {   // hybrid TMA + LSU gathers
+            if (a.seg == 2) return launch_pad<DT, 1, 2, 1, VEC>(a, map);
+            if (a.seg == 4) return a.nl >= 2 ? launch_pad<DT, 1, 4, 2, VEC>(a, map) : launch_pad<DT, 1, 4, 1, VEC>(a, map);
+            return launch_pad<DT, 1, 8, 4, VEC>(a, map);
+        }
+        if (a.seg == 8) return warps >= 2 ? launch_pad<DT, 2, 8, 0, VEC>(a, map) : launch_pad<DT, 1, 8, 0, VEC>(a, map);
         switch (warps) {
-            case 1: return launch_pad<DT, 1, 4, VEC>(a, map);
-            case 2: return launch_pad<DT, 2, 4, VEC>(a, map);
-            default: return launch_pad<DT, 4, 4, VEC>(a, map);
+            case 1: return launch_pad<DT, 1, 4, 0, VEC>(a, map);
+            case 2: return launch_pad<DT, 2, 4, 0, VEC>(a, map);
+            default: return launch_pad<DT, 4, 4, 0, VEC>(a, map);
         }
     }
     const bool tma = path == 2;
@@ -1599,9 +1760,18 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     if (g_force_path == 2 && tma_ok && make_bmap(&map, B, h->K, N, ldb, h->dtype)) path = 2;
     // TMA padded path: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB, else 512 B
     int seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : 4;
+    int nl = 0;
     {
         const char* e = getenv("DTC_PAD_SEG");
         if (e && atoi(e) == 4) seg = 4;
+        // hybrid (experiments): DTC_PAD_HYB=1 splits each CTA's columns half TMA, half LSU gathers
+        const char* hy = getenv("DTC_PAD_HYB");
+        if (hy && atoi(hy) == 1) {
+            const int64_t rb = N * elt;
+            if (rb >= 2048 && rb % 8 == 0) { seg = 8; nl = 4; }       // 1 KB TMA + 1 KB LSU per CTA
+            else if (rb >= 1024) { seg = 4; nl = 2; }                 // 512 B + 512 B
+            else { seg = 2; nl = 1; }                                 // 256 B + 256 B
+        }
     }
     if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg))
         path = 4;
@@ -1622,6 +1792,10 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
         const int slmax = (e && atoi(e) > 0) ? atoi(e) : 2;
         warps = nsl >= 4 && slmax >= 4 && seg == 4 ? 4 : (nsl >= 2 && slmax >= 2 ? 2 : 1);
         cta_cols = warps * slice_cols;
+        if (nl > 0) {
+            warps = 1;
+            cta_cols = slice_cols + nl * 256 / elt;
+        }
     }
     const int64_t gy64 = (N + cta_cols - 1) / cta_cols;
     if (gy64 > 65535) { set_error("N too large"); return DTC_ERR_UNSUPPORTED; }
@@ -1661,7 +1835,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
         pass_ws = (int)std::min<int64_t>(nws, std::max<int64_t>(1, fit));
         if (e && atoi(e) > 0) pass_ws = std::min(nws, atoi(e));
     }
-    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws, seg};
+    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws, seg, nl};
     cudaError_t e;
     if (h->dtype == DTC_FP16)
         e = use_vec ? dispatch<DTC_FP16, true>(warps, path, a, map) : dispatch<DTC_FP16, false>(warps, path, a, map);

@@ -16,13 +16,16 @@ from gpu_util import build, dev, spmm, check_tol
 
 pytestmark = pytest.mark.gpu
 
-PATHS = ["ldg", "tma", "dir", "pad"]
+PATHS = ["ldg", "tma", "dir", "pad", "hyb"]
 
 
 @pytest.fixture(params=PATHS)
-def path(request):
+def path(request, monkeypatch):
+    """hyb = the TMA path with half of every CTA's columns gathered by LSU warps (DTC_PAD_HYB)."""
     from paper_conf_asplos_fan0024_b200 import set_spmm_path
-    set_spmm_path(request.param)
+    if request.param == "hyb":
+        monkeypatch.setenv("DTC_PAD_HYB", "1")
+    set_spmm_path("pad" if request.param == "hyb" else request.param)
     yield request.param
     set_spmm_path("default")
 
