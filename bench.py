@@ -287,6 +287,9 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
         cfgd.update({"num_tc_blocks": T, "mean_nnz_tc": round(nnz / max(T, 1), 3), "sum_u": sum_u,
                      "unit_blocks": fmt.unit_blocks, "num_units": fmt.num_units,
                      "split_windows": fmt.num_split_windows})
+        # the paper's Selector, as a diagnostic: AR of one-CTA-per-window
+        sel = dtc.selector_ar(exp["row_window_offset"], torch.cuda.get_device_properties(0).multi_processor_count, 6)
+        cfgd["selector"] = {"ar": round(sel["ar"], 3), "occupancy": 6, "balanced_by_paper_rule": sel["ar"] > 1.2}
         kern_ms = statistics.mean(ms)
         achieved = lit / (kern_ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",

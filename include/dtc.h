@@ -171,6 +171,21 @@ void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory
 int dtc_tca_reorder(int64_t M, int64_t K, const int32_t* rowptr_host, const int32_t* colidx_host,
                     int32_t sm_num, int32_t* perm_host);
 
+/* ------------------------------------------------------------ Selector (NEXT-4, diagnostic)
+ * Simulation-based Selector, §4.5.2, Eq. (1), Fig. 10.  HOST, pure
+ * (no GPU needed).  rwo_host: RowWindowOffset int32[num_windows+1] (host copy, e.g.
+ * from dtc_format_export).  Simulates the base kernel (one thread block per window,
+ * length nTC_w) under the TB-scheduling model sm = 2(b mod S/2) + (floor(b/(S/2)) mod 2)
+ * (Eq. (1) with 64 -> S/2; reading C23) with `occupancy` resident blocks per
+ * SM, each SM running its blocks in index order on the first freed slot.  Outputs
+ * (each may be NULL): makespan_base = max over SMs of the last finish time (in TC
+ * blocks), makespan_balanced = NumTCBlocks / (num_sms * occupancy), ar = base /
+ * balanced (1 when T = 0).  The paper launches its balanced kernel when ar > 1.2;
+ * libdtc always runs TC-block-balanced units, so this is a report.
+ * Errors: INVALID (odd or < 2 num_sms, occupancy outside 1..1024, non-monotone rwo). */
+int dtc_selector_ar(const int32_t* rwo_host, int64_t num_windows, int32_t num_sms, int32_t occupancy,
+                    double* makespan_base, double* makespan_balanced, double* ar);
+
 /* ------------------------------------------------------------ distributed
  * One process per GPU (north_star).  Row windows are partitioned across ranks
  * into contiguous ranges balanced by TC-block count; every rank needs all of B,

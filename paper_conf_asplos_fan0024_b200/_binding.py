@@ -80,6 +80,7 @@ def lib():
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
+            L.dtc_selector_ar.argtypes = [_vp, _i64, _i32, _i32, _vp, _vp, _vp]
             L.dtc_tca_reorder.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp]
             L.dtc_nccl_unique_id.argtypes = [_vp]
             L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
@@ -295,6 +296,19 @@ def partition_windows(rwo, world: int) -> np.ndarray:
     _check(lib().dtc_partition_windows(rwo.ctypes.data_as(_vp), len(rwo) - 1, world, out.ctypes.data_as(_vp)),
            "dtc_partition_windows")
     return out
+
+
+def selector_ar(rwo, num_sms: int = 148, occupancy: int = 6) -> dict:
+    """Simulation-based Selector diagnostic (dtc_selector_ar): makespans of the
+    one-block-per-window kernel and of strict balance, and AR = their ratio (> 1.2: balance pays)."""
+    rwo = np.ascontiguousarray(rwo, dtype=np.int32)
+    out = np.zeros(3, dtype=np.float64)
+    a = out.ctypes.data
+    _check(lib().dtc_selector_ar(rwo.ctypes.data_as(_vp), len(rwo) - 1, num_sms, occupancy,
+                                 ctypes.c_void_p(a), ctypes.c_void_p(a + 8), ctypes.c_void_p(a + 16)),
+           "dtc_selector_ar")
+    return {"makespan_base": float(out[0]), "makespan_balanced": float(out[1]), "ar": float(out[2]),
+            "num_sms": num_sms, "occupancy": occupancy}
 
 
 def tca_reorder(M: int, K: int, rowptr, colidx, sm_num: int = 148) -> np.ndarray:
