@@ -171,6 +171,22 @@ void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory
 int dtc_tca_reorder(int64_t M, int64_t K, const int32_t* rowptr_host, const int32_t* colidx_host,
                     int32_t sm_num, int32_t* perm_host);
 
+/* ------------------------------------------------------------ GraphConv (NEXT-3)
+ * One GCN layer, §5.4 Eq. (2): Y = act((A x H) x W + b), in the
+ * paper's order: AH = A*H by dtc_spmm (this library's kernel), then the dense
+ * AH*W with bias and activation fused into a cuBLASLt TF32 GEMM epilogue (a plain
+ * library GEMM; FP32 accumulate).  All pointers device, row-major, dense:
+ *   H    K x F_in, dtype of the handle (fp32 for TF32 handles, fp16 for FP16);
+ *   W    F_in x F_out fp32;  bias F_out fp32 or NULL;  act DTC_ACT_NONE | DTC_ACT_RELU;
+ *   AH   M x F_in fp32, caller-owned workspace (holds A*H on return);
+ *   Y    M x F_out fp32, overwritten.
+ * Asynchronous on `stream`.  Errors: INVALID, UNSUPPORTED, OOM, CUDA. */
+typedef enum { DTC_ACT_NONE = 0, DTC_ACT_RELU = 1 } dtc_act_t;
+int dtc_graphconv(dtc_handle_t h, const void* H, int64_t F_in, const float* W, int64_t F_out,
+                  const float* bias, int32_t act, float* AH, float* Y, void* stream);
+/* Kernels one dtc_graphconv launches at least (SpMM + GEMM; cuBLASLt may add a reduction). */
+int dtc_graphconv_launches_per_call(void);
+
 /* ------------------------------------------------------------ Selector (NEXT-4, diagnostic)
  * Simulation-based Selector, §4.5.2, Eq. (1), Fig. 10.  HOST, pure
  * (no GPU needed).  rwo_host: RowWindowOffset int32[num_windows+1] (host copy, e.g.

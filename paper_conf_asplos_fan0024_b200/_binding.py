@@ -80,6 +80,8 @@ def lib():
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
+            L.dtc_graphconv.argtypes = [_vp, _vp, _i64, _vp, _i64, _vp, _i32, _vp, _vp, _vp]
+            L.dtc_graphconv_launches_per_call.argtypes = []
             L.dtc_selector_ar.argtypes = [_vp, _i64, _i32, _i32, _vp, _vp, _vp]
             L.dtc_tca_reorder.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp]
             L.dtc_nccl_unique_id.argtypes = [_vp]
@@ -255,6 +257,30 @@ class Format:
         _check(lib().dtc_spmm(self._h, _dptr(B), N, B.stride(0), _dptr(C), C.stride(0), _stream_ptr(stream)),
                "dtc_spmm")
         return C
+
+    def graphconv(self, H, W, bias=None, relu=True, AH=None, Y=None, stream=None):
+        """One GCN layer (dtc_graphconv, Eq. (2)): Y = act((A @ H) @ W + b).
+        H: CUDA K x F_in (handle dtype), W: CUDA fp32 F_in x F_out, bias fp32 F_out or None.
+        Returns (Y, AH); all tensors contiguous row-major."""
+        import torch
+        want = torch.float16 if self.dtype == "fp16" else torch.float32
+        if H.dtype != want or not H.is_cuda or not H.is_contiguous() or H.dim() != 2:
+            raise TypeError(f"H must be a contiguous 2-D CUDA {want} tensor")
+        F_in, F_out = H.shape[1], W.shape[1]
+        if W.dtype != torch.float32 or not W.is_contiguous() or W.shape[0] != F_in:
+            raise TypeError("W must be a contiguous fp32 (F_in x F_out) tensor")
+        if bias is not None and (bias.dtype != torch.float32 or bias.numel() != F_out or not bias.is_contiguous()):
+            raise TypeError("bias must be a contiguous fp32 tensor of F_out elements")
+        if AH is None:
+            AH = torch.empty((self.M, F_in), dtype=torch.float32, device=H.device)
+        if Y is None:
+            Y = torch.empty((self.M, F_out), dtype=torch.float32, device=H.device)
+        for t, shape in ((AH, (self.M, F_in)), (Y, (self.M, F_out))):
+            if t.dtype != torch.float32 or not t.is_contiguous() or tuple(t.shape) != shape:
+                raise TypeError(f"workspace/output must be contiguous fp32 {shape}")
+        _check(lib().dtc_graphconv(self._h, _dptr(H), F_in, _dptr(W), F_out, _dptr(bias), 1 if relu else 0,
+                                   _dptr(AH), _dptr(Y), _stream_ptr(stream)), "dtc_graphconv")
+        return Y, AH
 
     def spmm_raw(self, B_ptr: int, N: int, ldb: int, C_ptr: int, ldc: int, stream=None):
         _check(lib().dtc_spmm(self._h, B_ptr, N, ldb, C_ptr, ldc, _stream_ptr(stream)), "dtc_spmm")

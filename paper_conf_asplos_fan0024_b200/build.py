@@ -48,7 +48,7 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
            "-shared", "-Xcompiler", "-fPIC", "-cudart", "static",
            "-I", os.path.join(ROOT, "include"), "-I", inc,
            *[f"-D{d}" for d in defines], *sources(), "-o", target + ".tmp",
-           "-L", lib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + lib]
+           "-L", lib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + lib, "-lcublasLt"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)
