@@ -150,6 +150,14 @@ int dtc_spmm_launches_per_call(void);
  * (0 if it was the default), or DTC_ERR_INVALID for an unknown path. */
 int dtc_set_spmm_path(int path);
 
+/* Persistent launch of the padded-row path (path 4): on = 1 launches one wave of CTAs (resident
+ * CTAs per SM x SMs) that walk the F4 units in a static stride, the B ring and A batches of a CTA
+ * running across unit boundaries (no per-unit pipeline fill, no CTA launch per unit); on = 0
+ * launches one CTA per unit.  Same arithmetic and results either way (bit-identical: every unit
+ * is computed by one CTA in the same order).  Process-wide; DTC_PAD_PERS=0|1 sets the initial
+ * value.  Returns the previous setting. */
+int dtc_set_pad_persistent(int on);
+
 /* Diagnostics (the paper's per-SM busy/idle methodology, Fig. 3 P:152-160 / Fig. 15):
  * while enabled, each CTA of the TMA-path kernel writes 8 int64 to dev_buf[cta*8 ..]:
  * {cta, smid, t_start, t_first_issue, t_first_data, t_consumer_done, num_tc_blocks,

@@ -76,6 +76,7 @@ def lib():
             L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_launches_per_call.argtypes = []
             L.dtc_set_spmm_path.argtypes = [ctypes.c_int]
+            L.dtc_set_pad_persistent.argtypes = [ctypes.c_int]
             L.dtc_set_trace.argtypes = [_vp, _i64]
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
@@ -139,6 +140,11 @@ def set_trace(buf=None) -> None:
     if buf.dtype != torch.int64 or not buf.is_cuda or buf.dim() != 2 or buf.shape[1] != 8:
         raise TypeError("trace buffer must be a CUDA int64 tensor [ctas, 8]")
     _check(lib().dtc_set_trace(ctypes.c_void_p(buf.data_ptr()), buf.shape[0]), "dtc_set_trace")
+
+
+def set_pad_persistent(on: bool) -> bool:
+    """Persistent (one-wave) launch of the padded-row SpMM path (dtc_set_pad_persistent)."""
+    return bool(lib().dtc_set_pad_persistent(1 if on else 0))
 
 
 def set_spmm_path(path) -> int:

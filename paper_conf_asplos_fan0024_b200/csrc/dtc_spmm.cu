@@ -1169,7 +1169,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
            const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
-           int64_t ldb) {
+           int64_t ldb, int num_units) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1195,7 +1195,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     __shared__ int s_abyte[2];   // byte offset of the batch's first value inside its A slot
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const Unit u = units[blockIdx.x];
+    // Units of this CTA: blockIdx.x, blockIdx.x + gridDim.x, ... (one unit unless the launch is
+    // persistent).  The B ring and the A batches run on CTA-wide counters (gi0 blocks, gc0 batches
+    // before the current unit), so the producer keeps prefetching across unit boundaries.
     // CTA columns: SL TMA slices, then NL register-gather (LSU) warps of CW segments each (hybrid:
     // the TMA engine and the LSU pipe gather different columns of the same TC blocks concurrently)
     constexpr int CTA_COLS = SL * SLICE_COLS + NL * CW * COLW1;
@@ -1205,7 +1207,6 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int nsl = nsl64 < SL ? (int)(nsl64 > 0 ? nsl64 : 0) : SL;
     const int ncons = WPS * nsl;               // B-stage consumers
     const int nacons = ncons + NL;             // A-batch consumers
-    const int nblocks = u.be - u.bb;
     if (threadIdx.x == 0) {
         for (int i = 0; i < R; ++i) {
             mbar_init(&bar_full[i], 1);
@@ -1225,6 +1226,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
         const int32_t tcol = (int32_t)(col0 * ELT / pad_tma_elt<SEG>());  // TMA columns (4- or 8-byte elements)
         struct BatchMeta { int4 ids; int e0, e1; };
+        int gi0 = 0, gc0 = 0;
+        for (int ui = blockIdx.x; ui < num_units; ui += gridDim.x) {
+        const Unit u = units[ui];
+        const int nblocks = u.be - u.bb;
         auto meta_of = [&](int i0) -> BatchMeta {
             BatchMeta bm;
             const int i = i0 + jl;
@@ -1246,7 +1251,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         };
         BatchMeta cur = meta_of(0);
         for (int i0 = 0; i0 < nblocks; i0 += kPadBatch) {
-            const int c = i0 / kPadBatch, aslot = c & 1;
+            const int c = gc0 + i0 / kPadBatch, aslot = c & 1;
             const BatchMeta nxt = (i0 + kPadBatch < nblocks) ? meta_of(i0 + kPadBatch) : BatchMeta{make_int4(-1, -1, -1, -1), 0, 0};
             const int nj = min(kPadBatch, nblocks - i0);
             if (c >= 2) mbar_wait(&bar_aempty[aslot], ((c >> 1) - 1) & 1);
@@ -1272,7 +1277,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                              "r"(smem_u32(&bar_afull[aslot])) : "memory");
             }
             for (int j = 0; j < nj; ++j) {
-                const int i = i0 + j, s = i % R;
+                const int i = gi0 + i0 + j, s = i % R;
                 if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
                 if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
                 __syncwarp();
@@ -1292,8 +1297,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             }
             cur = nxt;
         }
+        gi0 += nblocks;
+        gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
+        }
         if (tr && lane == 0) {
-            tr[6] = nblocks;
+            tr[6] = gi0;
             tr[7] = gtimer();
         }
         return;
@@ -1307,7 +1315,6 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         const int64_t bcol = n0 + (int64_t)VW * g;
         const int64_t base = n0 + 2 * NJ1 * t;
         const int hoff = NJ1;
-        const bool split = u.split_id >= 0;
         const int pos = 8 * (g & 3) + 2 * t;
         const uint32_t below = (1u << pos) - 1u;
         const bool upper = g >= 4;
@@ -1322,6 +1329,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             v.w[0] = x.x; v.w[1] = x.y; v.w[2] = x.z; v.w[3] = x.w;
             return v;
         };
+        int gc0 = 0;
+        for (int ui = blockIdx.x; ui < num_units; ui += gridDim.x) {
+        const Unit u = units[ui];
+        const int nblocks = u.be - u.bb;
+        const bool split = u.split_id >= 0;
         float acc[NJ][4];
 #pragma unroll
         for (int jx = 0; jx < NJ; ++jx) acc[jx][0] = acc[jx][1] = acc[jx][2] = acc[jx][3] = 0.f;
@@ -1337,9 +1349,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         uint32_t vaddr = 0, maddr = 0, iaddr = 0, niaddr = 0;
         V16 b0[CW], b1[CW];
         if (nblocks > 0) {
-            mbar_wait(&bar_afull[0], 0);
-            const uint32_t slot = aring;
-            vaddr = slot + s_abyte[0];
+            mbar_wait(&bar_afull[gc0 & 1], (gc0 >> 1) & 1);
+            const uint32_t slot = aring + (gc0 & 1) * kPadASlot;
+            vaddr = slot + s_abyte[gc0 & 1];
             maddr = slot + kPadAValBytes;
             iaddr = niaddr = slot + kPadAIdsOff;
             const uint2 id = lds64(iaddr + 8 * t);
@@ -1347,7 +1359,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             for (int cw = 0; cw < CW; ++cw) { b0[cw] = gather((int)id.x, cw); b1[cw] = gather((int)id.y, cw); }
         }
         for (int i = 0; i < nblocks; ++i) {
-            const int j = i % kPadBatch, c = i / kPadBatch;
+            const int j = i % kPadBatch, c = gc0 + i / kPadBatch;
             // A fragment of block i (batch c)
             const uint4 m = lds128(maddr + j * 16);
             const uint32_t wl = upper ? m.y : m.x, wh = upper ? m.w : m.z;
@@ -1421,12 +1433,14 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
             }
         }
-        if (!active) return;
+        gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
+        if (!active) continue;
         if (!split) {
             while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         } else {
             int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
             split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+        }
         }
         return;
     }
@@ -1438,7 +1452,6 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int64_t n0 = col0 + (int64_t)warp * CW * COLW1;
     const int64_t base = n0 + (DT == DTC_TF32 ? 4 : 8) * t;
     const int hoff = DT == DTC_TF32 ? 16 : 32;
-    const bool split = u.split_id >= 0;
     const int pos = 8 * (g & 3) + 2 * t;
     const uint32_t below = (1u << pos) - 1u;
     const bool upper = g >= 4;
@@ -1447,6 +1460,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const uint32_t roff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + cg * 16;
     const uint32_t roff1 = roff0 + ODD;
 
+    int gi0 = 0, gc0 = 0;
+    for (int ui = blockIdx.x; ui < num_units; ui += gridDim.x) {
+    const Unit u = units[ui];
+    const int nblocks = u.be - u.bb;
+    const bool split = u.split_id >= 0;
     float acc[NJ][4];
 #pragma unroll
     for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
@@ -1461,7 +1479,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     }
     uint32_t vaddr = 0, maddr = 0;   // A batch: next block's first value (bytes), mask array
     for (int i = 0; i < nblocks; ++i) {
-        const int j = i % kPadBatch, c = i / kPadBatch;
+        const int j = i % kPadBatch, c = gc0 + i / kPadBatch;
         if (j == 0) {
             mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
             const uint32_t slot = aring + (c & 1) * kPadASlot;
@@ -1488,9 +1506,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         vaddr += ELT * (c01 + __popc(m.z) + __popc(m.w));
         // S2/S3: B fragments from the padded stage, mma
-        const int s = i % R;
-        mbar_wait(&bar_full[s], (i / R) & 1);
-        if (tr && i == 0 && threadIdx.x == 0) tr[4] = gtimer();
+        const int gi = gi0 + i, s = gi % R;
+        mbar_wait(&bar_full[s], (gi / R) & 1);
+        if (tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();
         const uint32_t st = ring + s * STAGE;
 #pragma unroll
         for (int cw = 0; cw < CW; ++cw) {
@@ -1533,6 +1551,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     } else {
         int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
         split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+    }
+    gi0 += nblocks;
+    gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
     }
     if (tr && threadIdx.x == 0) tr[5] = gtimer();
 }
@@ -1657,19 +1678,44 @@ static cudaError_t launch_dir(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
+// Persistent launch of the padded-row path (DTC_PAD_PERS=1 / dtc_set_pad_persistent): one wave of
+// CTAs (resident CTAs per SM x SMs, over the column groups), each walking units blockIdx.x,
+// blockIdx.x + gridDim.x, ... with its B ring running across unit boundaries.
+#ifndef DTC_PAD_PERS_DEFAULT
+#define DTC_PAD_PERS_DEFAULT 0
+#endif
+static int g_pad_pers = -1;
+static bool pad_persistent() {
+    if (g_pad_pers < 0) {
+        const char* e = getenv("DTC_PAD_PERS");
+        g_pad_pers = e ? (atoi(e) > 0 ? 1 : 0) : DTC_PAD_PERS_DEFAULT;
+    }
+    return g_pad_pers == 1;
+}
+
 template <int DT, int SL, int SEG, int NL, bool VEC>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     const size_t smem = pad_smem_bytes<SL, SEG>();
-    static bool attr = false;
-    if (!attr) {
+    constexpr int threads = (SL * SEG / 2 + NL + 1) * 32;
+    static int per_sm = 0;
+    if (!per_sm) {
         cudaFuncSetAttribute(k_spmm_pad<DT, SL, SEG, NL, VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = true;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_spmm_pad<DT, SL, SEG, NL, VEC>, threads, smem) !=
+                cudaSuccess || per_sm < 1) {
+            cudaGetLastError();
+            per_sm = 1;
+        }
     }
-    dim3 grid((unsigned)a.h->num_units, (unsigned)a.gy);
+    int64_t gx = a.h->num_units;
+    if (pad_persistent()) {
+        const int64_t slots = (int64_t)per_sm * num_sms();
+        gx = std::min<int64_t>(gx, std::max<int64_t>(1, slots / a.gy));
+    }
+    dim3 grid((unsigned)gx, (unsigned)a.gy);
     k_spmm_pad<DT, SL, SEG, NL, VEC><<<grid, (SL * SEG / 2 + NL + 1) * 32, smem, a.s>>>(
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
-        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb);
+        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units);
     return cudaGetLastError();
 }
 
@@ -1860,6 +1906,12 @@ extern "C" int dtc_set_trace(void* dev_buf, int64_t capacity_ctas) {
     g_trace = capacity_ctas ? reinterpret_cast<int64_t*>(dev_buf) : nullptr;
     g_trace_cap = capacity_ctas;
     return DTC_OK;
+}
+
+extern "C" int dtc_set_pad_persistent(int on) {
+    const int prev = pad_persistent() ? 1 : 0;
+    g_pad_pers = on > 0 ? 1 : 0;
+    return prev;
 }
 
 extern "C" int dtc_set_spmm_path(int path) {

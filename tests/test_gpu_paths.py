@@ -16,18 +16,22 @@ from gpu_util import build, dev, spmm, check_tol
 
 pytestmark = pytest.mark.gpu
 
-PATHS = ["ldg", "tma", "dir", "pad", "hyb"]
+PATHS = ["ldg", "tma", "dir", "pad", "hyb", "pers", "pershyb"]
 
 
 @pytest.fixture(params=PATHS)
 def path(request, monkeypatch):
-    """hyb = the TMA path with half of every CTA's columns gathered by LSU warps (DTC_PAD_HYB)."""
-    from paper_conf_asplos_fan0024_b200 import set_spmm_path
-    if request.param == "hyb":
+    """hyb = the TMA path with half of every CTA's columns gathered by LSU warps (DTC_PAD_HYB);
+    pers* = the padded-row path launched persistently (one wave walking the units)."""
+    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
+    p = request.param
+    if p.endswith("hyb"):
         monkeypatch.setenv("DTC_PAD_HYB", "1")
-    set_spmm_path("pad" if request.param == "hyb" else request.param)
-    yield request.param
+    prev = set_pad_persistent(p.startswith("pers"))
+    set_spmm_path("pad" if p in ("hyb", "pers", "pershyb") else p)
+    yield p
     set_spmm_path("default")
+    set_pad_persistent(prev)
 
 
 @pytest.mark.parametrize("dtype", ["tf32", "fp16"])
@@ -119,3 +123,25 @@ def test_row_perm_original_order(path):
     f = build(cfg.M, cfg.K, rp, ci, v, row_perm=dev(perm))
     Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v, B)
     assert np.array_equal(spmm(f, B).astype(np.float64), Cr)
+
+
+@pytest.mark.parametrize("name,U", [("c2", 0), ("c2", 16), ("c1", 2)])
+def test_persistent_bit_identical(name, U):
+    """Persistent and one-CTA-per-unit launches compute every unit in the same order."""
+    import torch
+    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg, cfg.N)
+    f = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U)
+    set_spmm_path("pad")
+    try:
+        prev = set_pad_persistent(False)
+        C0 = spmm(f, B)
+        set_pad_persistent(True)
+        C1 = spmm(f, B)
+        set_pad_persistent(prev)
+    finally:
+        set_spmm_path("default")
+    assert np.array_equal(C0, C1)
