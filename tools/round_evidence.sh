@@ -13,7 +13,14 @@ for c in c3 c3h c4 c5; do
   timeout 600 python bench.py --config $c --steps 30 --warmup 5 --no-cpu > gpurun_out/ev_bench_$c.json 2> gpurun_out/ev_bench_$c.err
 done
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_launches_c2.csv python bench.py --steps 5 --warmup 3 --no-cpu > /dev/null 2>&1
+# full ncu captures stay on the box (/tmp, tens of MB each); only text/CSV summaries come back
+mkdir -p /tmp/ncu
 for c in c2 c3 c3h c4 c5; do
-  timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_spmm -s 3 -c 1 -o gpurun_out/ev_prof_$c python bench.py --config $c --steps 3 --warmup 3 --minimal > /dev/null 2>&1
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_spmm -s 3 -c 1 -f -o /tmp/ncu/ev_prof_$c python bench.py --config $c --steps 3 --warmup 3 --minimal > gpurun_out/ev_ncu_$c.log 2>&1
+  python tools/ncu_summary.py /tmp/ncu/ev_prof_$c.ncu-rep > gpurun_out/ev_ncu_$c.txt 2>&1
+  ncu -i /tmp/ncu/ev_prof_$c.ncu-rep --page raw --csv > gpurun_out/ev_raw_$c.csv 2>/dev/null
   timeout 300 python tools/trace_cta.py $c > gpurun_out/ev_trace_$c.txt 2>&1
 done
+ncu -i /tmp/ncu/ev_prof_c2.ncu-rep --page source --csv > gpurun_out/ev_source_c2.csv 2>/dev/null
+du -sh gpurun_out
+find gpurun_out -size +16M -print -delete
