@@ -50,6 +50,9 @@ def parse_args():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--minimal", action="store_true", help="only the timed dtc loop (for ncu launch lists)")
+    p.add_argument("--graphconv", type=int, default=-1,
+                   help="also time one GraphConv layer (dtc_graphconv, NEXT-3) with F_in=N and this F_out "
+                        "(-1: F_out=N; 0: off)")
     return p.parse_args()
 
 
@@ -357,6 +360,24 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
                       "api": "dtc_spmm_dist (root H2D of B, NCCL broadcast, local kernel, per-rank C D2H)",
                       "steps": e2e_steps}
         out["format_build_ms"] = round(build_ms, 3)
+
+    # ---- GraphConv layer (NEXT-3, Eq. (2)): (A x H) x W + b, ReLU, with H = B
+    if args.graphconv != 0 and world == 1 and not args.minimal:
+        try:
+            F_out = N if args.graphconv < 0 else args.graphconv
+            Wg = torch.empty((N, F_out), dtype=torch.float32, device=dev).uniform_(-0.1, 0.1)
+            bg = torch.empty((F_out,), dtype=torch.float32, device=dev).uniform_(-0.1, 0.1)
+            AH = torch.empty((M, N), dtype=torch.float32, device=dev)
+            Yg = torch.empty((M, F_out), dtype=torch.float32, device=dev)
+            gsteps = max(5, min(args.steps, 50))
+            ms_g = time_loop(lambda: fmt.graphconv(B_d, Wg, bg, relu=True, AH=AH, Y=Yg), gsteps, 3, stream, flush)
+            gms = statistics.mean(ms_g)
+            out["graphconv"] = {"F_in": N, "F_out": F_out, "ms": round(gms, 5), "spmm_ms": round(kern_ms, 5),
+                                "dense_ms": round(gms - kern_ms, 5),
+                                "gflops_total": round((flops + 2.0 * M * N * F_out) / (gms * 1e-3) / 1e9, 1),
+                                "steps": gsteps, "api": "dtc_graphconv (DTC-SpMM + cuBLASLt TF32 bias/ReLU epilogue)"}
+        except Exception as e:  # noqa: BLE001
+            out["graphconv"] = {"error": str(e)}
 
     # ---- cuSPARSE on the same box (comparison system)
     if not args.no_cusparse and world == 1:

@@ -81,7 +81,7 @@ typedef struct {
     const int32_t* units;
 } dtc_format_view_t;
 
-/* Build options (zero-initialised = defaults).
+/* Build options (zero-initialised = defaults; window_order documented at the field).
  *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T, W and the SM count
  *   dedup_path   F1 per-window dedup: 0 auto, 1 force smem sort, 2 force chunked bitmap
  *                (both produce bit-identical formats; exposed for tests)
@@ -91,7 +91,9 @@ typedef struct {
     int32_t unit_blocks;
     int32_t dedup_path;
     int32_t guided;
-    int32_t reserved;
+    int32_t window_order;   /* F4 unit order: 0 = pieces of split windows first, then whole-window
+                               units (default; the split fixups overlap the launch instead of
+                               forming its tail), 1 = strict window order.  Same results. */
     /* optional row permutation (DEVICE int32[M], new row -> original row, a bijection):
      * the library condenses the permuted matrix and dtc_spmm still writes C in the
      * ORIGINAL row order (e.g. the TCA order from dtc_tca_reorder).  NULL = identity.

@@ -40,7 +40,7 @@ class _View(ctypes.Structure):
 
 
 class _Opts(ctypes.Structure):
-    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("reserved", _i32),
+    _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("window_order", _i32),
                 ("row_perm", _vp)]
 
 
@@ -202,7 +202,8 @@ class Format:
 
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
-              unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None) -> "Format":
+              unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None,
+              window_order: bool = False) -> "Format":
         """row_perm: optional CUDA int32 tensor [M], new row -> original row (e.g. tca_reorder);
         C is still produced in the original row order."""
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
@@ -211,7 +212,7 @@ class Format:
             import torch
             if row_perm.dtype != torch.int32 or not row_perm.is_cuda or row_perm.numel() != M:
                 raise TypeError("row_perm must be a CUDA int32 tensor of length M")
-        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), 0, _dptr(row_perm))
+        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value)

@@ -391,6 +391,19 @@ static Guide make_guide(int64_t T, int U, int64_t tail_span) {
     return g;
 }
 
+// Pieces of a split window (nb > U blocks): at least U blocks each, and at most ~sqrt(nb/2) of them.
+// A piece costs ~nb/np block times (~0.5 us each) and the last arriver's fixup chains np dependent
+// partial loads (~1 us each), so the window's critical path nb/np * 0.5 + np is smallest near
+// np = sqrt(nb/2) (c2's hub windows: ~1,600 blocks -> 29 pieces instead of 100 at U = 16).
+__host__ __device__ __forceinline__ int64_t split_pieces(int64_t nb, int64_t U) {
+    const int64_t byU = (nb + U - 1) / U;
+    int64_t r = (int64_t)sqrt((double)nb * 0.5);
+    if (r < 1) r = 1;
+    while (2 * r * r < nb) ++r;   // ceil(sqrt(nb/2))
+    while (r > 1 && 2 * (r - 1) * (r - 1) >= nb) --r;
+    return byU < r ? byU : r;
+}
+
 __global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, Guide gd,
                               int64_t* __restrict__ cnt, int64_t* __restrict__ split,
                               int64_t* __restrict__ slots) {
@@ -400,7 +413,7 @@ __global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, Guide 
         const bool big = nb > U;
         int64_t c;
         if (big) {
-            c = (nb + U - 1) / U;
+            c = split_pieces(nb, U);
         } else {
             bool starts = (w == 0);
             if (!starts) {
@@ -450,6 +463,24 @@ __global__ void k_units_fix(int64_t nu, int64_t W, const int32_t* __restrict__ r
     }
 }
 
+// Unit order: the pieces of split windows first (window order among them), then the whole-window
+// units (window order).  The last-arriving piece of a split window sums all its partials -- a chain
+// of npieces dependent loads -- so those units go first, where their fixups overlap the rest of the
+// launch instead of forming its tail (longest-processing-time-first).  Results do not depend on
+// the order (each unit is computed the same way; partials are summed in piece order).
+__global__ void k_units_flag(int64_t nu, const Unit* __restrict__ units, int64_t* __restrict__ flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nu; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = units[i].split_id >= 0 ? 1 : 0;
+}
+__global__ void k_units_permute(int64_t nu, const Unit* __restrict__ in, const int64_t* __restrict__ pos,
+                                Unit* __restrict__ out) {
+    const int64_t nsu = pos[nu];
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nu; i += (int64_t)gridDim.x * blockDim.x) {
+        const bool sp = in[i].split_id >= 0;
+        out[sp ? pos[i] : nsu + (i - pos[i])] = in[i];
+    }
+}
+
 // ---------------------------------------------------------------- host driver
 static unsigned grid_for(int64_t work, int per_block, int cap = 1 << 20) {
     int64_t g = (work + per_block - 1) / per_block;
@@ -462,7 +493,7 @@ static void free_format(dtc_format* h, cudaStream_t s) {
     if (!h) return;
     dfree(h->rwo, s); dfree(h->tco, s); dfree(h->lid, s); dfree(h->atob, s);
     dfree(h->vals, s); dfree(h->mask, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
-    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s);
+    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s);
 }
 
 struct BuildTemps {
@@ -685,6 +716,21 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             TRY(dalloc(&h->units, std::max<int64_t>(h->num_units, 1), s));
             k_units_fill<<<grid_for(W, 256, 4096), 256, 0, s>>>(W, h->rwo, gd, t.ucnt, t.usplit, t.uslots, h->units);
             k_units_fix<<<grid_for(h->num_units, 256, 4096), 256, 0, s>>>(h->num_units, W, h->rwo, h->units);
+            if (h->num_split > 0 && !(opts && opts->window_order)) {
+                const int64_t nu = h->num_units;
+                int64_t* pos = nullptr;
+                Unit* sorted = nullptr;
+                TRY(dalloc(&pos, nu + 1, s));
+                TRY(dalloc(&sorted, nu, s));
+                dfree(t.scan_tmp, s);
+                TRY(dalloc(&t.scan_tmp, scan_tmp_elems(nu + 1) + 64, s));
+                k_units_flag<<<grid_for(nu, 256, 4096), 256, 0, s>>>(nu, h->units, pos);
+                exclusive_scan_i64(pos, pos, nu, t.scan_tmp, s);
+                k_units_permute<<<grid_for(nu, 256, 4096), 256, 0, s>>>(nu, h->units, pos, sorted);
+                dfree(h->units, s);
+                dfree(pos, s);
+                h->units = sorted;
+            }
         }
         TRYC(cudaGetLastError());
         st.mark("F4 units");

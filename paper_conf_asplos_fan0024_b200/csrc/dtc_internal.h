@@ -56,6 +56,9 @@ struct dtc_format {
     size_t stage_C_bytes = 0;
     // optional row map (row of the condensed matrix -> row of C), from dtc_build_opts_t.row_perm
     int32_t* rowmap = nullptr;
+    // persistent padded-row launch: dynamic unit counters, 2 per column group (self-resetting)
+    int32_t* uctr = nullptr;
+    int64_t uctr_len = 0;
     // GraphConv (dtc_graphconv): cuBLASLt workspace for the dense (A*H)*W step
     uint8_t* gemm_ws = nullptr;
     size_t gemm_ws_bytes = 0;

@@ -275,6 +275,7 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
     __threadfence();
 #pragma unroll
     for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+#pragma unroll 2
     for (int pc = 0; pc < u.npieces; ++pc) {
         const int64_t sl = (int64_t)u.slot_base + pc;
 #pragma unroll
@@ -1169,7 +1170,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
            const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
-           int64_t ldb, int num_units) {
+           int64_t ldb, int num_units, int32_t* __restrict__ uctr) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1191,13 +1192,17 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
     const uint32_t aring = ring + R * STAGE;                          // [2][kPadASlot] A batches
-    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[2], bar_aempty[2];
+    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[2], bar_aempty[2], bar_ufull[2], bar_uempty[2];
     __shared__ int s_abyte[2];   // byte offset of the batch's first value inside its A slot
+    __shared__ int s_unit[2][10];   // published unit: Unit record, end block of its first window, index (-1 = done)
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    // Units of this CTA: blockIdx.x, blockIdx.x + gridDim.x, ... (one unit unless the launch is
-    // persistent).  The B ring and the A batches run on CTA-wide counters (gi0 blocks, gc0 batches
-    // before the current unit), so the producer keeps prefetching across unit boundaries.
+    // Units of this CTA: blockIdx.x only (one CTA per unit), or -- persistent launch -- the units
+    // the producer draws from the column group's atomic counter uctr[2*blockIdx.y] (dynamic
+    // balance; the last CTA resets it), or blockIdx.x + k*gridDim.x when uctr is null.  The
+    // producer publishes each unit (record + end of its first window) to the consumers through
+    // s_unit / bar_ufull / bar_uempty; the B ring and the A batches run on CTA-wide counters
+    // (gi0 blocks, gc0 batches before the current unit), so prefetching continues across units.
     // CTA columns: SL TMA slices, then NL register-gather (LSU) warps of CW segments each (hybrid:
     // the TMA engine and the LSU pipe gather different columns of the same TC blocks concurrently)
     constexpr int CTA_COLS = SL * SLICE_COLS + NL * CW * COLW1;
@@ -1215,6 +1220,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         for (int i = 0; i < 2; ++i) {
             mbar_init(&bar_afull[i], 1);
             mbar_init(&bar_aempty[i], nacons);
+            mbar_init(&bar_ufull[i], 1);
+            mbar_init(&bar_uempty[i], ncons);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -1225,34 +1232,76 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         const uint32_t tx = (uint32_t)nsl * pad_tx_bytes<SEG>();
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
         const int32_t tcol = (int32_t)(col0 * ELT / pad_tma_elt<SEG>());  // TMA columns (4- or 8-byte elements)
+        // Batch metadata is loaded one batch ahead -- across unit boundaries, with the next unit's
+        // record loaded one unit ahead -- and only shuffled into gather4 row order when its batch
+        // starts, so no load latency sits between two batches (or two units) of TMA issues.
+        struct Raw { int4 mine; int e0, e1; };
         struct BatchMeta { int4 ids; int e0, e1; };
-        int gi0 = 0, gc0 = 0;
-        for (int ui = blockIdx.x; ui < num_units; ui += gridDim.x) {
-        const Unit u = units[ui];
-        const int nblocks = u.be - u.bb;
-        auto meta_of = [&](int i0) -> BatchMeta {
-            BatchMeta bm;
-            const int i = i0 + jl;
-            const int4 mine = i < nblocks ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(u.bb + i) * 8) + half)
-                                          : make_int4(-1, -1, -1, -1);
-            int4 o;   // partner's half
-            o.x = __shfl_xor_sync(0xffffffffu, mine.x, 1);
-            o.y = __shfl_xor_sync(0xffffffffu, mine.y, 1);
-            o.z = __shfl_xor_sync(0xffffffffu, mine.z, 1);
-            o.w = __shfl_xor_sync(0xffffffffu, mine.w, 1);
-            bm.ids = half == 0 ? make_int4(mine.x, mine.z, o.x, o.z)     // rows 0, 2, 4, 6
-                               : make_int4(o.y, o.w, mine.y, mine.w);    // rows 1, 3, 5, 7
-            bm.e0 = bm.e1 = 0;
-            if (lane == 0 && i0 < nblocks) {
-                bm.e0 = __ldg(tco + u.bb + i0);
-                bm.e1 = __ldg(tco + u.bb + min(i0 + kPadBatch, nblocks));
+        auto load_raw = [&](const Unit& uu, int i0) -> Raw {
+            Raw r;
+            const int nbu = uu.be - uu.bb, i = i0 + jl;
+            r.mine = i < nbu ? __ldg(reinterpret_cast<const int4*>(atob + (int64_t)(uu.bb + i) * 8) + half)
+                             : make_int4(-1, -1, -1, -1);
+            r.e0 = r.e1 = 0;
+            if (lane == 0 && i0 < nbu) {
+                r.e0 = __ldg(tco + uu.bb + i0);
+                r.e1 = __ldg(tco + uu.bb + min(i0 + kPadBatch, nbu));
             }
+            return r;
+        };
+        auto finish = [&](const Raw& r) -> BatchMeta {
+            BatchMeta bm;
+            int4 o;   // partner's half
+            o.x = __shfl_xor_sync(0xffffffffu, r.mine.x, 1);
+            o.y = __shfl_xor_sync(0xffffffffu, r.mine.y, 1);
+            o.z = __shfl_xor_sync(0xffffffffu, r.mine.z, 1);
+            o.w = __shfl_xor_sync(0xffffffffu, r.mine.w, 1);
+            bm.ids = half == 0 ? make_int4(r.mine.x, r.mine.z, o.x, o.z)     // rows 0, 2, 4, 6
+                               : make_int4(o.y, o.w, r.mine.y, r.mine.w);    // rows 1, 3, 5, 7
+            bm.e0 = r.e0;
+            bm.e1 = r.e1;
             return bm;
         };
-        BatchMeta cur = meta_of(0);
+        const Unit kNone = {0, 0, 0, 0, -1, 0, 0, 0};
+        auto first_end = [&](const Unit& uu) -> int {
+            return (uu.split_id < 0 && uu.wb < uu.we) ? __ldg(rwo + uu.wb + 1) : INT_MAX;
+        };
+        int32_t* const myctr = uctr ? uctr + 2 * blockIdx.y : nullptr;
+        int kst = 0;   // static ordinal
+        auto draw = [&]() -> int {   // next unit index (lane 0's value in dynamic mode: shuffle before use)
+            if (myctr) return lane == 0 ? atomicAdd(myctr, 1) : 0;
+            if (gridDim.x == num_units) return kst++ == 0 ? (int)blockIdx.x : num_units;
+            return (int)blockIdx.x + (kst++) * (int)gridDim.x;
+        };
+        auto bcast = [&](int v) -> int { return myctr ? __shfl_sync(0xffffffffu, v, 0) : v; };
+        int q0 = draw();
+        int q1 = draw();
+        q0 = bcast(q0);
+        q1 = bcast(q1);
+        Unit u = q0 < num_units ? units[q0] : kNone;
+        Unit un = q1 < num_units ? units[q1] : kNone;
+        int end0 = first_end(u), end0n = INT_MAX;
+        Raw rnext = load_raw(u, 0);
+        int gi0 = 0, gc0 = 0;
+        for (int ord = 0;; ++ord) {
+        // publish unit ord to the consumers (index -1 = no more units)
+        if (ord >= 2) mbar_wait(&bar_uempty[ord & 1], ((ord >> 1) - 1) & 1);
+        if (lane == 0) {
+            int* su = s_unit[ord & 1];
+            su[0] = u.wb; su[1] = u.we; su[2] = u.bb; su[3] = u.be;
+            su[4] = u.split_id; su[5] = u.piece; su[6] = u.npieces; su[7] = u.slot_base;
+            su[8] = end0;
+            su[9] = q0 < num_units ? q0 : -1;
+            mbar_arrive(&bar_ufull[ord & 1]);
+        }
+        if (q0 >= num_units) break;
+        const int q2 = draw();   // reserve the unit after next now; its latency hides behind this unit
+        const int nblocks = u.be - u.bb;
         for (int i0 = 0; i0 < nblocks; i0 += kPadBatch) {
             const int c = gc0 + i0 / kPadBatch, aslot = c & 1;
-            const BatchMeta nxt = (i0 + kPadBatch < nblocks) ? meta_of(i0 + kPadBatch) : BatchMeta{make_int4(-1, -1, -1, -1), 0, 0};
+            const BatchMeta cur = finish(rnext);
+            rnext = i0 + kPadBatch < nblocks ? load_raw(u, i0 + kPadBatch) : load_raw(un, 0);
+            if (i0 == 0) end0n = first_end(un);
             const int nj = min(kPadBatch, nblocks - i0);
             if (c >= 2) mbar_wait(&bar_aempty[aslot], ((c >> 1) - 1) & 1);
             if (lane == 0) {
@@ -1295,10 +1344,25 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 }
                 __syncwarp();
             }
-            cur = nxt;
+        }
+        if (nblocks == 0) {
+            rnext = load_raw(un, 0);
+            end0n = first_end(un);
         }
         gi0 += nblocks;
         gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
+        q0 = q1;
+        u = un;
+        end0 = end0n;
+        q1 = bcast(q2);
+        un = q1 < num_units ? units[q1] : kNone;
+        }
+        if (myctr && lane == 0) {   // the last CTA of the column group resets its counter
+            __threadfence();
+            if (atomicAdd(myctr + 1, 1) == (int)gridDim.x - 1) {
+                atomicExch(myctr, 0);
+                atomicExch(myctr + 1, 0);
+            }
         }
         if (tr && lane == 0) {
             tr[6] = gi0;
@@ -1460,9 +1524,23 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const uint32_t roff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + cg * 16;
     const uint32_t roff1 = roff0 + ODD;
 
+    // Units arrive from the producer (s_unit), record and first-window end already loaded, so a
+    // unit boundary costs no dependent global load.
     int gi0 = 0, gc0 = 0;
-    for (int ui = blockIdx.x; ui < num_units; ui += gridDim.x) {
-    const Unit u = units[ui];
+    for (int ord = 0;; ++ord) {
+    mbar_wait(&bar_ufull[ord & 1], (ord >> 1) & 1);
+    Unit u;
+    int end0, uidx;
+    {
+        const int* su = s_unit[ord & 1];
+        u.wb = su[0]; u.we = su[1]; u.bb = su[2]; u.be = su[3];
+        u.split_id = su[4]; u.piece = su[5]; u.npieces = su[6]; u.slot_base = su[7];
+        end0 = su[8];
+        uidx = su[9];
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&bar_uempty[ord & 1]);
+    if (uidx < 0) break;
     const int nblocks = u.be - u.bb;
     const bool split = u.split_id >= 0;
     float acc[NJ][4];
@@ -1471,11 +1549,13 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     int cur = u.wb;
     int next_end = INT_MAX;
     if (!split) {
-        while (cur < u.we && rwo[cur + 1] <= u.bb) {
+        int e = end0;
+        while (cur < u.we && e <= u.bb) {   // leading empty windows
             store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
             ++cur;
+            e = cur < u.we ? rwo[cur + 1] : INT_MAX;
         }
-        next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+        next_end = cur < u.we ? e : INT_MAX;
     }
     uint32_t vaddr = 0, maddr = 0;   // A batch: next block's first value (bytes), mask array
     for (int i = 0; i < nblocks; ++i) {
@@ -1534,6 +1614,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             mbar_arrive(&bar_empty[s]);
             if (j == kPadBatch - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[c & 1]);
         }
+
         if (u.bb + i + 1 == next_end) {
             store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
 #pragma unroll
@@ -1707,15 +1788,30 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
         }
     }
     int64_t gx = a.h->num_units;
+    int32_t* uctr = nullptr;
     if (pad_persistent()) {
         const int64_t slots = (int64_t)per_sm * num_sms();
         gx = std::min<int64_t>(gx, std::max<int64_t>(1, slots / a.gy));
+        // dynamic unit counters (one pair per column group, self-resetting); the hybrid LSU warps
+        // walk a static stride, so NL > 0 stays static
+        if (NL == 0 && gx < a.h->num_units) {
+            if (a.h->uctr_len < 2 * a.gy) {
+                dfree(a.h->uctr, a.s);
+                a.h->uctr_len = 0;
+                if (dalloc(&a.h->uctr, (size_t)2 * a.gy, a.s) != DTC_OK) return cudaErrorMemoryAllocation;
+                cudaError_t e = cudaMemsetAsync(a.h->uctr, 0, sizeof(int32_t) * 2 * a.gy, a.s);
+                if (e != cudaSuccess) return e;
+                a.h->uctr_len = 2 * a.gy;
+            }
+            uctr = a.h->uctr;
+        }
     }
     dim3 grid((unsigned)gx, (unsigned)a.gy);
     k_spmm_pad<DT, SL, SEG, NL, VEC><<<grid, (SL * SEG / 2 + NL + 1) * 32, smem, a.s>>>(
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
-        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units);
+        (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units,
+        uctr);
     return cudaGetLastError();
 }
 

@@ -145,3 +145,26 @@ def test_persistent_bit_identical(name, U):
     finally:
         set_spmm_path("default")
     assert np.array_equal(C0, C1)
+
+
+@pytest.mark.parametrize("name,U", [("c2", 16), ("c1", 2)])
+def test_unit_order_split_first(name, U):
+    """F4 default order: split-window pieces first (window order), then whole-window units;
+    same units as strict window order and the same C bit for bit."""
+    from gpu_util import check_units
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg, cfg.N)
+    f0 = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U)
+    f1 = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U, window_order=True)
+    e0, e1 = f0.export(), f1.export()
+    check_units(e0, cfg.M)
+    u0, u1 = e0["units"], e1["units"]
+    assert sorted(map(tuple, u0)) == sorted(map(tuple, u1))
+    sp = u0[:, 4] >= 0
+    k = int(sp.sum())
+    assert k > 0 and np.all(sp[:k]) and not np.any(sp[k:])
+    assert np.all(np.diff(u0[:k, 2]) >= 0) and np.all(np.diff(u0[k:, 2]) >= 0)   # window (block) order inside
+    assert np.all(np.diff(u1[:, 2]) >= 0)
+    assert np.array_equal(spmm(f0, B), spmm(f1, B))
