@@ -242,13 +242,24 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
     }
 }
 
-// Split-window fixup for one warp's tile (deterministic: slots summed in piece order).
-template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
-__device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
-                                            int32_t* __restrict__ ctr, float* __restrict__ C, int64_t ldc, int64_t M,
-                                            int64_t N, int g, int lane, int64_t base, int hoff,
-                                            const int32_t* __restrict__ rowmap) {
-    const int64_t slot = (int64_t)u.slot_base + u.piece;
+// Split-window fixup for one warp's tile, deterministic, two levels.  A window split into np
+// pieces forms groups of G = ceil(sqrt(np)) consecutive pieces (one group when np <= 4).  Every piece
+// writes its partial to its slot; the last arriving piece of a group sums the group's slots in piece
+// order (into the group's first slot); the last arriving group sums the group sums in group order
+// and stores C.  The chain of dependent partial loads is G + np/G instead of np (the single-level
+// chain made the last arriver of a hub window the tail of the launch).  Counters live at
+// ctr0[slot * cstride] (one per slot and warp column slice): group g at its first slot, the window
+// at slot_base + 1 (never a group's first slot when there are >= 2 groups); all self-resetting.
+__device__ __forceinline__ int fixup_group(int np) {
+    if (np <= 4) return np;
+    int g = 1;
+    while (g * g < np) ++g;
+    return g;
+}
+
+template <int NJ, int QPC, int CSTRIDE>
+__device__ __forceinline__ void fixup_write(float (&acc)[NJ][4], float* __restrict__ ws, int64_t slot, int64_t npad,
+                                            int g, int64_t base, int hoff) {
 #pragma unroll
     for (int half = 0; half < 2; ++half) {
         float* prow = ws + (slot * kWindow + g + 8 * half) * npad;
@@ -262,22 +273,17 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
                                    acc[4 * q + 2][2 * half + hi], acc[4 * q + 3][2 * half + hi]));
             }
     }
-    __threadfence();
-    __syncwarp();
-    int last = 0;
-    if (lane == 0) {
-        const int prev = atomicAdd(ctr, 1);
-        last = (prev == u.npieces - 1);
-        if (last) *ctr = 0;  // self-reset for the next launch (stream-ordered)
-    }
-    last = __shfl_sync(0xffffffffu, last, 0);
-    if (!last) return;
-    __threadfence();
+}
+
+// acc := sum over k < cnt of slot (s0 + k * step), in k order
+template <int NJ, int QPC, int CSTRIDE>
+__device__ __forceinline__ void fixup_sum(float (&acc)[NJ][4], const float* __restrict__ ws, int64_t s0, int64_t step,
+                                          int cnt, int64_t npad, int g, int64_t base, int hoff) {
 #pragma unroll
     for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
-#pragma unroll 2
-    for (int pc = 0; pc < u.npieces; ++pc) {
-        const int64_t sl = (int64_t)u.slot_base + pc;
+#pragma unroll 1
+    for (int k = 0; k < cnt; ++k) {
+        const int64_t sl = s0 + k * step;
 #pragma unroll
         for (int half = 0; half < 2; ++half) {
             const float* prow = ws + (sl * kWindow + g + 8 * half) * npad;
@@ -293,6 +299,39 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
                     acc[4 * q + 3][2 * half + hi] += v.w;
                 }
         }
+    }
+}
+
+// true in every lane of the warp that arrives n-th at *ctr (the counter is reset for the next launch)
+__device__ __forceinline__ bool arrive_last(int32_t* ctr, int n, int lane) {
+    __threadfence();
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) {
+        const int prev = atomicAdd(ctr, 1);
+        last = (prev == n - 1);
+        if (last) *ctr = 0;
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (last) __threadfence();
+    return last != 0;
+}
+
+template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
+__device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
+                                            int32_t* __restrict__ ctr0, int64_t cstride, float* __restrict__ C,
+                                            int64_t ldc, int64_t M, int64_t N, int g, int lane, int64_t base, int hoff,
+                                            const int32_t* __restrict__ rowmap) {
+    const int np = u.npieces, G = fixup_group(np);
+    const int g0 = (u.piece / G) * G, gn = min(G, np - g0), ngr = (np + G - 1) / G;
+    const int64_t sb = u.slot_base;
+    fixup_write<NJ, QPC, CSTRIDE>(acc, ws, sb + u.piece, npad, g, base, hoff);
+    if (!arrive_last(ctr0 + (sb + g0) * cstride, gn, lane)) return;
+    fixup_sum<NJ, QPC, CSTRIDE>(acc, ws, sb + g0, 1, gn, npad, g, base, hoff);
+    if (ngr > 1) {
+        fixup_write<NJ, QPC, CSTRIDE>(acc, ws, sb + g0, npad, g, base, hoff);
+        if (!arrive_last(ctr0 + (sb + 1) * cstride, ngr, lane)) return;
+        fixup_sum<NJ, QPC, CSTRIDE>(acc, ws, sb, G, ngr, npad, g, base, hoff);
     }
     store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, u.wb, g, base, hoff, acc, false, rowmap);
 }
@@ -512,8 +551,8 @@ k_spmm_tma(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         return;
     }
     // S5: split-window fixup per consumer warp
-    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+    split_fixup<NJ, VEC>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp, (int64_t)gridDim.y * 8, C, ldc, M, N, g,
+                         lane, base, hoff, rowmap);
 }
 
 // ============================================================ fallback: register gather
@@ -828,8 +867,8 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         return;
     }
-    int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp, (int64_t)gridDim.y * 8, C,
+                                     ldc, M, N, g, lane, base, hoff, rowmap);
 }
 
 // ============================================================ direct path (no shared memory)
@@ -1069,8 +1108,8 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
         while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         return;
     }
-    int32_t* ctr = counters + (int64_t)u.split_id * nws + wsl;
-    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+    split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + wsl, (int64_t)nws, C, ldc, M, N, g, lane, base, hoff,
+                                     rowmap);
 }
 
 // ============================================================ TMA path with padded rows (path 4)
@@ -1093,14 +1132,12 @@ k_spmm_dir(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
 // elements, box 132) or 8 (1 KB slices, 8-byte TMA elements, box 130 -- one gather4 op moves
 // 2x the bytes, for B rows of >= 1 KB).  Row pitch SEG*128 + 16 (= 16 mod 128).
 template <int SEG> constexpr int pad_row_bytes() { return SEG * 128 + 16; }
-template <int SEG> constexpr int pad_box_elts() { return SEG == 2 ? 68 : (SEG == 4 ? 132 : 130); }
-template <int SEG> constexpr int pad_tma_elt() { return SEG == 8 ? 8 : 4; }
 template <int SEG> constexpr int pad_odd_off() { return (4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_slice_bytes() { return (pad_odd_off<SEG>() + 4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_tx_bytes() { return 8 * pad_row_bytes<SEG>(); }
 static_assert(pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16, "row pitch must be 16 mod 128");
-static_assert(pad_box_elts<4>() * 4 == pad_row_bytes<4>() && pad_box_elts<8>() * 8 == pad_row_bytes<8>() &&
-                  pad_box_elts<2>() * 4 == pad_row_bytes<2>() && pad_row_bytes<2>() % 128 == 16, "box");
+static_assert(pad_row_bytes<2>() % 128 == 16 && pad_row_bytes<2>() % 8 == 0 && pad_row_bytes<4>() % 8 == 0 &&
+                  pad_row_bytes<8>() % 8 == 0, "row pitch must be 16 mod 128 and whole 8-byte elements");
 template <int SL>
 constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
@@ -1170,7 +1207,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
            const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
-           int64_t ldb, int num_units, int32_t* __restrict__ uctr) {
+           int64_t ldb, int num_units, int32_t* __restrict__ uctr, int te) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1231,7 +1268,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         // ================= producer: A batches (bulk copies) + B gather4 (4 rows x one slice per op)
         const uint32_t tx = (uint32_t)nsl * pad_tx_bytes<SEG>();
         const int half = lane & 1, jl = lane >> 1;     // lane pair (2j, 2j+1): even / odd rows of block i0 + j
-        const int32_t tcol = (int32_t)(col0 * ELT / pad_tma_elt<SEG>());  // TMA columns (4- or 8-byte elements)
+        const int32_t tcol = (int32_t)(col0 * ELT / te);  // TMA columns (te = 4- or 8-byte elements)
+        const int32_t tslice = SEG * 128 / te;             // TMA columns per slice
         // Batch metadata is loaded one batch ahead -- across unit boundaries, with the next unit's
         // record loaded one unit ahead -- and only shuffled into gather4 row order when its batch
         // starts, so no load latency sits between two batches (or two units) of TMA issues.
@@ -1337,7 +1375,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                         asm volatile(
                             "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                             " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-                            "l"(&bmap), "r"(tcol + sl * (SEG * 128 / pad_tma_elt<SEG>())), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
+                            "l"(&bmap), "r"(tcol + sl * tslice), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
                             "r"(cur.ids.w), "r"(smem_u32(&bar_full[s]))
                             : "memory");
                     }
@@ -1502,8 +1540,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (!split) {
             while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
         } else {
-            int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-            split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+            split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp, (int64_t)gridDim.y * 8,
+                                             C, ldc, M, N, g, lane, base, hoff, rowmap);
         }
         }
         return;
@@ -1630,8 +1668,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     if (!split) {
         while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
     } else {
-        int32_t* ctr = counters + ((int64_t)u.split_id * gridDim.y + blockIdx.y) * 8 + warp;
-        split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, ctr, C, ldc, M, N, g, lane, base, hoff, rowmap);
+        split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp, (int64_t)gridDim.y * 8, C,
+                                         ldc, M, N, g, lane, base, hoff, rowmap);
     }
     gi0 += nblocks;
     gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
@@ -1675,14 +1713,24 @@ static bool make_bmap(CUtensorMap* map, const void* B, int64_t K, int64_t N, int
 
 // Tensor map of B viewed as 4-byte elements (fp16 pairs for FP16): K rows x N*elt/4 columns,
 // gather4 boxes of kPadBoxElts x 1, no swizzle (rows land 528 bytes apart, see k_spmm_pad).
-static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype, int seg) {
+// TMA element size of the padded path: 8 bytes whenever a B row is a whole number of 8-byte words
+// (half the elements per gather4 op of 4-byte elements), else 4 (DTC_PAD_TE=4 forces 4).
+static int pad_te(int64_t N, int dtype, int seg) {
+    const char* e = getenv("DTC_PAD_TE");
+    if (e && atoi(e) == 4 && seg != 8) return 4;
+    return ((N * elt_size(dtype)) % 8 == 0) ? 8 : 4;
+}
+
+static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N, int64_t ldb, int dtype, int seg,
+                          int te) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return false;
     const int elt = elt_size(dtype);
-    const int te = seg == 8 ? 8 : 4;   // TMA element bytes
+    if (seg == 8 && te != 8) return false;
+    const int row_bytes = seg == 2 ? pad_row_bytes<2>() : seg == 4 ? pad_row_bytes<4>() : pad_row_bytes<8>();
     cuuint64_t dims[2] = {(cuuint64_t)(N * elt / te), (cuuint64_t)K};
     cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
-    cuuint32_t box[2] = {(cuuint32_t)(seg == 2 ? pad_box_elts<2>() : seg == 4 ? pad_box_elts<4>() : pad_box_elts<8>()), 1};
+    cuuint32_t box[2] = {(cuuint32_t)(row_bytes / te), 1};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(map, te == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2,
                      const_cast<void*>(B), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -1706,6 +1754,7 @@ struct LaunchArgs {
     int nws, pass_ws;   // direct path: warp slices of N, slices per L2-resident pass
     int seg;            // TMA padded path: 128-byte segments per slice (2, 4 or 8)
     int nl;             // TMA padded path: register-gather (LSU) warps per CTA (hybrid), 0 = none
+    int te;             // TMA padded path: TMA element bytes (4 or 8)
 };
 
 template <int DT, int WARPS>
@@ -1811,7 +1860,7 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
         (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units,
-        uctr);
+        uctr, a.te);
     return cudaGetLastError();
 }
 
@@ -1915,7 +1964,8 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
             else { seg = 2; nl = 1; }                                 // 256 B + 256 B
         }
     }
-    if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg))
+    const int te = pad_te(N, h->dtype, seg);
+    if (g_force_path == 4 && tma_ok && (N * elt) % 4 == 0 && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg, te))
         path = 4;
     // columns per warp: the 128B-swizzled TMA path one 128-byte slice per warp, the others two
     const int colw_tma = h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW;
@@ -1944,7 +1994,8 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     const int gy = (int)gy64;
     const int64_t npad = gy64 * cta_cols;
     if (h->num_split > 0) {
-        const int64_t ncnt = h->num_split * gy * 8;   // per (split, column group, consumer warp)
+        // per (slot, column group, consumer warp) -- or (slot, warp slice) on the direct path
+        const int64_t ncnt = h->num_slots * std::max<int64_t>((int64_t)gy * 8, need);
         if (ncnt > h->counters_len) {
             dfree(h->counters, s);
             h->counters_len = 0;
@@ -1977,7 +2028,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
         pass_ws = (int)std::min<int64_t>(nws, std::max<int64_t>(1, fit));
         if (e && atoi(e) > 0) pass_ws = std::min(nws, atoi(e));
     }
-    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws, seg, nl};
+    LaunchArgs a{h, B, ldb, C, ldc, N, gy, npad, s, nws, pass_ws, seg, nl, te};
     cudaError_t e;
     if (h->dtype == DTC_FP16)
         e = use_vec ? dispatch<DTC_FP16, true>(warps, path, a, map) : dispatch<DTC_FP16, false>(warps, path, a, map);

@@ -79,3 +79,19 @@ def test_product_path_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".h", ".cuh", ".cpp")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in src.replace("no oracle", ""), f
+
+
+def test_default_spmm_kernels_do_not_spill():
+    """The padded-row kernels dtc_spmm launches by default (vector C path, no hybrid warps) keep
+    everything in registers: no stack frame (spills would sit on the per-block critical path)."""
+    out = subprocess.run(["cuobjdump", "-res-usage", dtc.library_path()], capture_output=True, text=True).stdout
+    lines = out.splitlines()
+    seen = 0
+    for i, line in enumerate(lines):
+        m = re.search(r"Function (_ZN3dtc10k_spmm_padILi\d+ELi\d+ELi\d+ELi0ELb1E\S*):", line)
+        if m:
+            seen += 1
+            stack = int(re.search(r"STACK:(\d+)", lines[i + 1]).group(1))
+            local = int(re.search(r"LOCAL:(\d+)", lines[i + 1]).group(1))
+            assert stack == 0 and local == 0, (m.group(1)[:60], lines[i + 1])
+    assert seen >= 6
