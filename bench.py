@@ -50,6 +50,9 @@ def parse_args():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--minimal", action="store_true", help="only the timed dtc loop (for ncu launch lists)")
+    p.add_argument("--tca", type=int, default=-1,
+                   help="also time the SpMM on the TCA-reordered matrix (NEXT-1, dtc_tca_reorder + row_perm; "
+                        "C still in the original order): 1 on, 0 off, -1 on when nnz < 10M")
     p.add_argument("--graphconv", type=int, default=-1,
                    help="also time one GraphConv layer (dtc_graphconv, NEXT-3) with F_in=N and this F_out "
                         "(-1: F_out=N; 0: off)")
@@ -360,6 +363,27 @@ def run_dtc(args, cfg, N, rank, world, local_rank):
                       "api": "dtc_spmm_dist (root H2D of B, NCCL broadcast, local kernel, per-rank C D2H)",
                       "steps": e2e_steps}
         out["format_build_ms"] = round(build_ms, 3)
+
+    # ---- TCA reordering (NEXT-1, Alg. 1): host preprocessing, then the same kernel on
+    # the permuted ME-TCF (rows permuted inside the library, C written in the original row order)
+    if (args.tca == 1 or (args.tca < 0 and nnz < 10_000_000)) and world == 1 and not args.minimal:
+        try:
+            t0 = time.perf_counter()
+            perm = dtc.tca_reorder(M, K, rp, ci, torch.cuda.get_device_properties(dev).multi_processor_count)
+            reorder_s = time.perf_counter() - t0
+            perm_d = torch.from_numpy(perm).to(dev)
+            fmt_t = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks,
+                                     guided=args.guided, row_perm=perm_d)
+            C_t = torch.empty((M, N), dtype=torch.float32, device=dev)
+            ms_t = time_loop(lambda: fmt_t.spmm(B_d, C_t), max(10, min(args.steps, 100)), 3, stream, flush)
+            tms = statistics.mean(ms_t)
+            out["tca"] = {"value": round(flops / (tms * 1e-3) / 1e9, 2), "unit": UNIT, "ms_per_step": round(tms, 5),
+                          "num_tc_blocks": fmt_t.num_tc_blocks, "mean_nnz_tc": round(nnz / max(fmt_t.num_tc_blocks, 1), 3),
+                          "reorder_host_s": round(reorder_s, 3), "speedup_vs_unordered": round(kern_ms / tms, 3),
+                          "matches_unordered": bool(torch.allclose(C_t, C_d, rtol=1e-2, atol=1e-2))}
+            fmt_t.close()
+        except Exception as e:  # noqa: BLE001
+            out["tca"] = {"error": str(e)}
 
     # ---- GraphConv layer (NEXT-3, Eq. (2)): (A x H) x W + b, ReLU, with H = B
     if args.graphconv != 0 and world == 1 and not args.minimal:

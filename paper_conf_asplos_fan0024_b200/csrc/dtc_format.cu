@@ -524,13 +524,15 @@ struct BuildTemps {
 
 // F4 unit size: ~2 windows' worth of TC blocks, clamped to [64, 256] (measured sweep for the
 // TMA path, profiles/r01_design_evidence.md: arxiv-like 64, banded 64-128, products-like 128,
-// reddit-like >= 256), and small enough that there are at least 2 units per SM.
+// reddit-like >= 256), and small enough for >= 4 waves of 6 CTAs per SM (so the last partial wave
+// is a small part of the launch: arxiv-like T = 115k -> U = 32, +3% measured over U = 64 in three
+// runs); never below 16.
 static int auto_unit_blocks(int64_t T, int64_t W) {
     int64_t target = W > 0 ? (2 * T) / W : 64;
     if (target < 64) target = 64;
     if (target > 256) target = 256;
-    const int64_t cap = T / (2 * (int64_t)num_sms());
-    if (target > cap) target = cap < 8 ? 8 : cap;
+    const int64_t cap = T / (24 * (int64_t)num_sms());
+    if (target > cap) target = cap < 16 ? 16 : cap;
     return (int)target;
 }
 
