@@ -228,6 +228,8 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
                 if (VEC) {
 #if defined(DTC_L2_HINTS) && (DTC_L2_HINTS & 2)
                     if (c < N) stg_hint(crow + c, v, l2_policy_first());
+#elif defined(DTC_C_STORE_CS)
+                    if (c < N) __stcs(reinterpret_cast<float4*>(crow + c), v);   // streaming (evict-first)
 #else
                     if (c < N) *reinterpret_cast<float4*>(crow + c) = v;
 #endif
@@ -1207,7 +1209,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
            const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
-           int64_t ldb, int num_units, int32_t* __restrict__ uctr, int te) {
+           int64_t ldb, int num_units, int32_t* __restrict__ uctr, int te, int lsur) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1366,9 +1368,39 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             for (int j = 0; j < nj; ++j) {
                 const int i = gi0 + i0 + j, s = i % R;
                 if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
+                if (tr && i == 0 && lane == 0) tr[3] = gtimer();
+                if (lsur > 0 && i % lsur == lsur - 1) {
+                    // dual-engine gather: this block's rows go through the LSU path (cp.async 16 B
+                    // per lane-chunk, zero-filled for -1 ids and past N) into the same padded stage,
+                    // tracked by the stage's mbarrier -- the TMA unit is the per-SM limit otherwise
+                    const int r = lane >> 2, srcl = 2 * j + (r & 1);
+                    const int ix = __shfl_sync(0xffffffffu, cur.ids.x, srcl), iy = __shfl_sync(0xffffffffu, cur.ids.y, srcl);
+                    const int iz = __shfl_sync(0xffffffffu, cur.ids.z, srcl), iw = __shfl_sync(0xffffffffu, cur.ids.w, srcl);
+                    const int q = r >> 1;
+                    const int id = q == 0 ? ix : q == 1 ? iy : q == 2 ? iz : iw;
+                    const char* srow = reinterpret_cast<const char*>(B) + (int64_t)(id < 0 ? 0 : id) * ldb * ELT;
+                    const int64_t rowb = N * ELT;
+                    for (int sl = 0; sl < nsl; ++sl) {
+                        const uint32_t dst = ring + s * STAGE + sl * SLB + (r & 1) * ODD + q * ROWB;
+                        const int64_t cb = col0 * ELT + (int64_t)sl * SEG * 128;
+#pragma unroll
+                        for (int k = 0; k < 2 * SEG; ++k) {
+                            const int ch = (lane & 3) + 4 * k;
+                            const int64_t off = cb + ch * 16;
+                            const int64_t rem = rowb - off;
+                            const uint32_t n = id < 0 ? 0u : (rem >= 16 ? 16u : (rem > 0 ? (uint32_t)rem : 0u));
+                            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst + ch * 16),
+                                         "l"(n ? srow + off : reinterpret_cast<const char*>(B)), "r"(n) : "memory");
+                        }
+                    }
+                    asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(smem_u32(&bar_full[s])) : "memory");
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&bar_full[s]);
+                    __syncwarp();
+                    continue;
+                }
                 if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
                 __syncwarp();
-                if (tr && i == 0 && lane == 0) tr[3] = gtimer();
                 if (jl == j) {
                     for (int sl = 0; sl < nsl; ++sl) {
                         const uint32_t dst = ring + s * STAGE + sl * SLB + half * ODD;
@@ -1823,6 +1855,16 @@ static bool pad_persistent() {
     return g_pad_pers == 1;
 }
 
+// Dual-engine gather (DTC_PAD_LSU=k): every k-th TC block of a CTA is gathered by the producer warp
+// with cp.async (LSU path) instead of TMA gather4; 0 = TMA only.
+#ifndef DTC_PAD_LSU_DEFAULT
+#define DTC_PAD_LSU_DEFAULT 0
+#endif
+static int pad_lsu_every() {   // read per launch (experiments flip it between calls)
+    const char* e = getenv("DTC_PAD_LSU");
+    return e ? std::max(0, atoi(e)) : DTC_PAD_LSU_DEFAULT;
+}
+
 template <int DT, int SL, int SEG, int NL, bool VEC>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     const size_t smem = pad_smem_bytes<SL, SEG>();
@@ -1860,7 +1902,7 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
         map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
         (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units,
-        uctr, a.te);
+        uctr, a.te, pad_lsu_every());
     return cudaGetLastError();
 }
 

@@ -16,7 +16,7 @@ from gpu_util import build, dev, spmm, check_tol
 
 pytestmark = pytest.mark.gpu
 
-PATHS = ["ldg", "tma", "dir", "pad", "hyb", "pers", "pershyb"]
+PATHS = ["ldg", "tma", "dir", "pad", "hyb", "pers", "pershyb", "lsu2", "lsu3", "perslsu3"]
 
 
 @pytest.fixture(params=PATHS)
@@ -27,8 +27,10 @@ def path(request, monkeypatch):
     p = request.param
     if p.endswith("hyb"):
         monkeypatch.setenv("DTC_PAD_HYB", "1")
+    if "lsu" in p:   # dual-engine gather: every k-th block by cp.async
+        monkeypatch.setenv("DTC_PAD_LSU", p[-1])
     prev = set_pad_persistent(p.startswith("pers"))
-    set_spmm_path("pad" if p in ("hyb", "pers", "pershyb") else p)
+    set_spmm_path("pad" if (p in ("hyb", "pers", "pershyb") or "lsu" in p) else p)
     yield p
     set_spmm_path("default")
     set_pad_persistent(prev)
