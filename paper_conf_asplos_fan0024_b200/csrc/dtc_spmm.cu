@@ -1151,10 +1151,14 @@ constexpr int pad_stages() {
 // A side of the TMA path: per batch of kPadBatch TC blocks, one bulk copy of the (16-byte
 // aligned superset of the) batch's TCValues -- contiguous, TCOffset[b0] .. TCOffset[b0+16] --
 // and one of its 16 occupancy masks, double buffered.
-constexpr int kPadBatch = 16;
-constexpr int kPadAValBytes = 8320;               // >= 16 blocks x 128 values x 4 B + 16, 128-aligned
-constexpr int kPadAIdsOff = kPadAValBytes + 256;  // + 16 masks
-constexpr int kPadASlot = kPadAIdsOff + 512;       // + 16 x 8 SparseAtoB ids (hybrid LDG warps)
+#ifndef DTC_PAD_BATCH
+#define DTC_PAD_BATCH 16
+#endif
+constexpr int kPadBatch = DTC_PAD_BATCH;
+constexpr int kPadAValBytes = kPadBatch * 512 + 128;       // >= batch x 128 values x 4 B + 16, 128-aligned
+constexpr int kPadAIdsOff = kPadAValBytes + kPadBatch * 16;  // + one 16-byte mask per block
+constexpr int kPadASlot = kPadAIdsOff + kPadBatch * 32;      // + 8 SparseAtoB ids per block (hybrid LDG warps)
+static_assert(kPadBatch >= 1 && kPadBatch <= 16, "batch: the producer's lane pairs hold one block each");
 template <int SL, int SEG>
 constexpr size_t pad_smem_bytes_() { return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * kPadASlot + 128; }
 template <int SL, int SEG>
