@@ -170,3 +170,30 @@ def test_unit_order_split_first(name, U):
     assert np.all(np.diff(u0[:k, 2]) >= 0) and np.all(np.diff(u0[k:, 2]) >= 0)   # window (block) order inside
     assert np.all(np.diff(u1[:, 2]) >= 0)
     assert np.array_equal(spmm(f0, B), spmm(f1, B))
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("N", [1024, 1100, 2048])
+def test_persistent_many_column_groups(dtype, N):
+    """Wide B (several CTA column groups, each with its own dynamic unit counter), split windows:
+    persistent == one-CTA-per-unit bit for bit, and within tolerance of the oracle."""
+    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
+    M, K = 600, 500
+    rp, ci = datagen.random_csr(M, K, 0.08, N)
+    v = datagen.uniform(N, 1, len(ci))
+    B = datagen.uniform(N, 2, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype, unit_blocks=4)
+    set_spmm_path("pad")
+    try:
+        prev = set_pad_persistent(False)
+        C0 = spmm(f, B)
+        set_pad_persistent(True)
+        C1 = spmm(f, B)
+        C2 = spmm(f, B)       # counters reset by the previous launch
+        set_pad_persistent(prev)
+    finally:
+        set_spmm_path("default")
+    assert np.array_equal(C0, C1) and np.array_equal(C1, C2)
+    check_tol(C1, M, K, rp, ci, v, B, dtype)
