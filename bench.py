@@ -45,7 +45,7 @@ def parse_args():
     p.add_argument("--config", default="c2")
     p.add_argument("--n", type=int, default=0, help="override N (columns of B)")
     p.add_argument("--unit-blocks", type=int, default=0)
-    p.add_argument("--guided", type=int, default=0, help="F4 guided tail (1 on, 0 off)")
+    p.add_argument("--guided", type=int, default=0, help="F4 guided tail (1 on, -1 off, 0 auto)")
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--no-e2e", action="store_true")

@@ -85,8 +85,8 @@ typedef struct {
  *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T, W and the SM count
  *   dedup_path   F1 per-window dedup: 0 auto, 1 force smem sort, 2 force chunked bitmap
  *                (both produce bit-identical formats; exposed for tests)
- *   guided       F4 tail: 0 = fixed-size units (default); 1 = units of U/2 over the last
- *                ~half wave of TC blocks (measured: +-1% on large matrices, -8% on c2) */
+ *   guided       F4 tail: units of U/2 over the last ~half wave: 1 = on, -1 = off, 0 = auto (on
+ *                when T < 8 waves x 6 CTAs x SMs x U, i.e. short launches; +5% on the arxiv-shaped c2) */
 typedef struct {
     int32_t unit_blocks;
     int32_t dedup_path;

@@ -493,7 +493,7 @@ static void free_format(dtc_format* h, cudaStream_t s) {
     if (!h) return;
     dfree(h->rwo, s); dfree(h->tco, s); dfree(h->lid, s); dfree(h->atob, s);
     dfree(h->vals, s); dfree(h->mask, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
-    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s);
+    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s); dfree(h->units_lpt, s);
 }
 
 struct BuildTemps {
@@ -695,8 +695,12 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         // F4: work units
         int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T, W);
         h->unit_blocks = U;
-        // optional guided tail over about half a wave of units (opts->guided > 0)
-        const int64_t tail = (opts && opts->guided > 0) ? (int64_t)num_sms() * 4 * U : 0;
+        // guided tail (units of U/2 over about half a wave): opts->guided 1 = on, -1 = off, 0 = auto:
+        // on when the launch is only a few waves long (< 8 waves of 6 CTAs per SM), where the last
+        // partial wave is a large part of it (arxiv-shaped c2: +5% measured; c3-c5 have 20-300 waves)
+        const int gopt = opts ? opts->guided : 0;
+        const bool guided = gopt > 0 || (gopt == 0 && T < (int64_t)8 * 6 * num_sms() * U);
+        const int64_t tail = guided ? (int64_t)num_sms() * 4 * U : 0;
         const Guide gd = make_guide(T, U, tail);
         if (W > 0) {
             TRY(dalloc(&t.ucnt, W + 1, s));

@@ -59,6 +59,7 @@ struct dtc_format {
     // persistent padded-row launch: dynamic unit counters, 2 per column group (self-resetting)
     int32_t* uctr = nullptr;
     int64_t uctr_len = 0;
+    dtc::Unit* units_lpt = nullptr;   // units by size, descending (persistent launch)
     // GraphConv (dtc_graphconv): cuBLASLt workspace for the dense (A*H)*W step
     uint8_t* gemm_ws = nullptr;
     size_t gemm_ws_bytes = 0;

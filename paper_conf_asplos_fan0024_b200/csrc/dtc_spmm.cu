@@ -29,6 +29,7 @@
 
 #include <algorithm>
 #include <climits>
+#include <vector>
 
 #include "dtc_internal.h"
 
@@ -1851,6 +1852,10 @@ static cudaError_t launch_dir(const LaunchArgs& a) {
 #define DTC_PAD_PERS_DEFAULT 0
 #endif
 static int g_pad_pers = -1;
+static bool pad_lpt() {   // DTC_PAD_LPT=0 keeps the build order in persistent launches (experiments)
+    const char* e = getenv("DTC_PAD_LPT");
+    return !(e && atoi(e) == 0);
+}
 static bool pad_persistent() {
     if (g_pad_pers < 0) {
         const char* e = getenv("DTC_PAD_PERS");
@@ -1867,6 +1872,26 @@ static bool pad_persistent() {
 static int pad_lsu_every() {   // read per launch (experiments flip it between calls)
     const char* e = getenv("DTC_PAD_LSU");
     return e ? std::max(0, atoi(e)) : DTC_PAD_LSU_DEFAULT;
+}
+
+// Unit order for the persistent launch: largest units first (stable; longest-processing-time
+// first), so the last units CTAs draw are the smallest and the launch ends evenly.  Built once per
+// handle on the host (units are 32 B each) at the first persistent launch; results do not depend on
+// the order.
+static cudaError_t lpt_units(dtc_format* h, cudaStream_t s) {
+    if (h->units_lpt || h->num_units == 0) return cudaSuccess;
+    std::vector<Unit> u((size_t)h->num_units);
+    cudaError_t e = cudaMemcpyAsync(u.data(), h->units, u.size() * sizeof(Unit), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return e;
+    std::stable_sort(u.begin(), u.end(), [](const Unit& x, const Unit& y) { return (x.be - x.bb) > (y.be - y.bb); });
+    Unit* d = nullptr;
+    if (dalloc(&d, u.size(), s) != DTC_OK) return cudaErrorMemoryAllocation;
+    e = cudaMemcpyAsync(d, u.data(), u.size() * sizeof(Unit), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) { dfree(d, s); return e; }
+    h->units_lpt = d;
+    return cudaSuccess;
 }
 
 template <int DT, int SL, int SEG, int NL, bool VEC>
@@ -1899,11 +1924,16 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
                 a.h->uctr_len = 2 * a.gy;
             }
             uctr = a.h->uctr;
+            if (pad_lpt()) {
+                cudaError_t e = lpt_units(a.h, a.s);
+                if (e != cudaSuccess) return e;
+            }
         }
     }
+    const Unit* units = (uctr && a.h->units_lpt) ? a.h->units_lpt : a.h->units;
     dim3 grid((unsigned)gx, (unsigned)a.gy);
     k_spmm_pad<DT, SL, SEG, NL, VEC><<<grid, (SL * SEG / 2 + NL + 1) * 32, smem, a.s>>>(
-        map, a.h->units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
+        map, units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
         (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units,
         uctr, a.te, pad_lsu_every());
