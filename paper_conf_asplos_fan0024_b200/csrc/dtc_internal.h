@@ -54,6 +54,10 @@ struct dtc_format {
     size_t stage_B_bytes = 0;
     float* stage_C = nullptr;
     size_t stage_C_bytes = 0;
+    // host-API copy pipeline (dtc_spmm_host with column chunks): copy-in / copy-out streams and
+    // per-chunk events, created on first use
+    cudaStream_t hstream[2] = {nullptr, nullptr};
+    cudaEvent_t hev[2 * 16 + 1] = {};
     // optional row map (row of the condensed matrix -> row of C), from dtc_build_opts_t.row_perm
     int32_t* rowmap = nullptr;
     // persistent padded-row launch: dynamic unit counters, 2 per column group (self-resetting)

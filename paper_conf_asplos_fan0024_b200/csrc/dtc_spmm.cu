@@ -2144,6 +2144,23 @@ extern "C" int dtc_set_spmm_path(int path) {
     return prev;
 }
 
+// Column chunks for dtc_spmm_host: C(:, cols) depends only on B(:, cols), so the call is pipelined
+// over column chunks -- H2D of chunk j+1 runs while chunk j computes and its C chunk goes back
+// (PCIe / C2C are full duplex).  Every output element is the same sum in the same order as one
+// dtc_spmm over all N columns (the kernels' per-column arithmetic does not depend on N).
+// Pitched copies of narrow row pieces run well below the wide-copy rate, and each chunk's kernel
+// re-reads the format, so chunks stay >= 256 B of a B row (>= 512 B when rows are wider than 512 B),
+// at most 4 (measured on B200, dtc_spmm_host e2e: c2 2 chunks +24%, c3 2 chunks +27%, c5 4 chunks
+// +58%; 128-256 B chunks of wide rows were slower than no pipelining, profiles/r01_host_chunks.txt).
+// DTC_HOST_CHUNKS overrides the count (1 = the unpipelined copy-in, kernel, copy-out sequence).
+static int host_chunks(int64_t N, int elt, size_t bytes) {
+    const int64_t row = N * elt;
+    int64_t c = row < 256 ? 1 : row <= 512 ? 2 : std::min<int64_t>(4, row / 512);
+    if (bytes < ((size_t)8 << 20)) c = 1;   // small calls: latency, not bandwidth
+    if (const char* e = getenv("DTC_HOST_CHUNKS")) c = atoi(e);
+    return (int)std::max<int64_t>(1, std::min<int64_t>({c, 16, (N + 31) / 32}));   // widths: multiples of 32 columns
+}
+
 extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                              int64_t ldc, void* stream) {
     if (!h || !C_host || (!B_host && h->K > 0)) { set_error("null argument"); return DTC_ERR_INVALID; }
@@ -2172,13 +2189,55 @@ extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int6
         }
         h->stage_C_bytes = cbytes;
     }
-    if (h->K > 0)
-        DTC_CUDA(cudaMemcpy2DAsync(h->stage_B, N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice, s));
-    int rc = spmm_launch(h, h->stage_B, N, N, h->stage_C, N, s);
-    if (rc) return rc;
-    if (h->M > 0)
-        DTC_CUDA(cudaMemcpy2DAsync(C_host, ldc * sizeof(float), h->stage_C, N * sizeof(float), N * sizeof(float), h->M,
-                                   cudaMemcpyDeviceToHost, s));
+    const int nch = host_chunks(N, elt, bbytes + cbytes);
+    if (nch <= 1) {
+        if (h->K > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(h->stage_B, N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice, s));
+        int rc = spmm_launch(h, h->stage_B, N, N, h->stage_C, N, s);
+        if (rc) return rc;
+        if (h->M > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(C_host, ldc * sizeof(float), h->stage_C, N * sizeof(float), N * sizeof(float),
+                                       h->M, cudaMemcpyDeviceToHost, s));
+        DTC_CUDA(cudaStreamSynchronize(s));
+        return DTC_OK;
+    }
+    for (auto& hs : h->hstream)
+        if (!hs) DTC_CUDA(cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking));
+    for (auto& e : h->hev)
+        if (!e) DTC_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    cudaStream_t sin = h->hstream[0], sout = h->hstream[1];
+    cudaEvent_t* evb = h->hev;         // [nch] chunk j of B resident
+    cudaEvent_t* evk = h->hev + 16;    // [nch] chunk j of C computed
+    cudaEvent_t evs = h->hev[32];      // start / end fence
+    // the copy streams start after everything already queued on s (e.g. staging reallocation)
+    DTC_CUDA(cudaEventRecord(evs, s));
+    DTC_CUDA(cudaStreamWaitEvent(sin, evs, 0));
+    DTC_CUDA(cudaStreamWaitEvent(sout, evs, 0));
+    // chunk widths: multiples of 32 columns, the remainder spread over the first chunks
+    const int64_t units32 = (N + 31) / 32;
+    int64_t c0 = 0;
+    uint8_t* sb = reinterpret_cast<uint8_t*>(h->stage_B);
+    for (int j = 0; j < nch; ++j) {
+        const int64_t u = units32 / nch + (j < units32 % nch ? 1 : 0);
+        const int64_t nc = std::min<int64_t>(N - c0, u * 32);
+        uint8_t* bj = sb + (size_t)h->K * c0 * elt;                 // K x nc, ldb = nc
+        float* cj = h->stage_C + (size_t)h->M * c0;                   // M x nc, ldc = nc
+        if (h->K > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(bj, nc * elt, reinterpret_cast<const uint8_t*>(B_host) + c0 * elt, ldb * elt,
+                                       nc * elt, h->K, cudaMemcpyHostToDevice, sin));
+        DTC_CUDA(cudaEventRecord(evb[j], sin));
+        DTC_CUDA(cudaStreamWaitEvent(s, evb[j], 0));
+        int rc = spmm_launch(h, bj, nc, nc, cj, nc, s);
+        if (rc) return rc;
+        DTC_CUDA(cudaEventRecord(evk[j], s));
+        DTC_CUDA(cudaStreamWaitEvent(sout, evk[j], 0));
+        if (h->M > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(C_host + c0, ldc * sizeof(float), cj, nc * sizeof(float), nc * sizeof(float),
+                                       h->M, cudaMemcpyDeviceToHost, sout));
+        c0 += nc;
+    }
+    DTC_CUDA(cudaEventRecord(evs, sout));
+    DTC_CUDA(cudaStreamWaitEvent(s, evs, 0));
     DTC_CUDA(cudaStreamSynchronize(s));
     return DTC_OK;
 }

@@ -235,3 +235,26 @@ def test_p2_integer_full_size_sampled_exact(name, N):
     Cr, Bd = oracle.spmm_at(cfg.M, rp, ci, v.astype(np.float32), B.astype(np.float32), rows, cols)
     assert float(Bd.max()) < 2 ** 23
     assert np.array_equal(C[rows, cols].astype(np.float64), Cr)
+
+
+@pytest.mark.parametrize("chunks", ["1", "2", "3", "4", "16"])
+@pytest.mark.parametrize("dtype,N", [("tf32", 128), ("tf32", 100), ("tf32", 257), ("fp16", 192)])
+def test_host_api_column_chunks(chunks, dtype, N, monkeypatch):
+    """dtc_spmm_host pipelined over column chunks (DTC_HOST_CHUNKS): C(:, cols) depends only on
+    B(:, cols), so every chunking returns what one dtc_spmm over all N columns returns (the
+    per-column sum order is the same), and it stays within the O1 tolerance."""
+    monkeypatch.setenv("DTC_HOST_CHUNKS", chunks)
+    M, K = 3000, 2500
+    rp, ci = datagen.random_csr(M, K, 0.01, N + 7)
+    v = datagen.uniform(N, 3, len(ci))
+    B = datagen.uniform(N, 4, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    Cd = spmm(f, B)
+    Ch = f.spmm_host(np.ascontiguousarray(B))
+    check_tol(Ch, M, K, rp, ci, v, B, dtype)
+    assert np.array_equal(Cd, Ch)
+    # a second call reuses the staging buffers, streams and events
+    Ch2 = f.spmm_host(np.ascontiguousarray(B))
+    assert np.array_equal(Ch, Ch2)
