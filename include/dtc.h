@@ -136,8 +136,9 @@ int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, float* C, in
  * ldc) and synchronises `stream`.  Pinned host memory gives full PCIe/C2C rate.
  * Calls of >= 8 MB are pipelined over column chunks (C(:, cols) depends only on B(:, cols)):
  * the copy-in of chunk j+1 overlaps chunk j's kernel and copy-out on library-owned streams;
- * the result is bit-identical to one dtc_spmm over all N columns.  Chunks: 2 for B rows of
- * 256-512 B, rows/512 B (<= 4) for wider rows; DTC_HOST_CHUNKS=k overrides (1 = unpipelined). */
+ * the result is bit-identical to one dtc_spmm over all N columns.  Chunks: up to 4, each >= 512 B
+ * of a B row (>= 256 B when the format is smaller than B); DTC_HOST_CHUNKS=k overrides
+ * (1 = unpipelined). */
 int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                   int64_t ldc, void* stream);
 

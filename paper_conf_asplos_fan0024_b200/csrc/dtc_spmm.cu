@@ -2149,13 +2149,17 @@ extern "C" int dtc_set_spmm_path(int path) {
 // (PCIe / C2C are full duplex).  Every output element is the same sum in the same order as one
 // dtc_spmm over all N columns (the kernels' per-column arithmetic does not depend on N).
 // Pitched copies of narrow row pieces run well below the wide-copy rate, and each chunk's kernel
-// re-reads the format, so chunks stay >= 256 B of a B row (>= 512 B when rows are wider than 512 B),
-// at most 4 (measured on B200, dtc_spmm_host e2e: c2 2 chunks +24%, c3 2 chunks +27%, c5 4 chunks
-// +58%; 128-256 B chunks of wide rows were slower than no pipelining, profiles/r01_host_chunks.txt).
+// re-reads the format (A), so chunks keep >= 512 B of a B row, or >= 256 B when the format is
+// smaller than B (the kernels are short next to the copies); at most 4 chunks.  Measured on B200,
+// dtc_spmm_host e2e (profiles/r01_host_chunks.txt): c2 2 x 256 B +24%, c4 2 x 256 B +27%, c3 2 x 512 B
+// +27%, c5 4 x 512 B +58%; c3h (FP16, format 5x B) 2 x 256 B -12%, so it stays unpipelined.
 // DTC_HOST_CHUNKS overrides the count (1 = the unpipelined copy-in, kernel, copy-out sequence).
-static int host_chunks(int64_t N, int elt, size_t bytes) {
+static int host_chunks(const dtc_format* h, int64_t N, int elt, size_t bytes) {
     const int64_t row = N * elt;
-    int64_t c = row < 256 ? 1 : row <= 512 ? 2 : std::min<int64_t>(4, row / 512);
+    const double fmt_bytes = (double)h->nnz * (elt + 1) + 36.0 * (double)h->T + 4.0 * (double)h->W;
+    const double b_bytes = (double)std::max<int64_t>(h->K, 1) * row;
+    const int64_t wmin = fmt_bytes < b_bytes ? 256 : 512;
+    int64_t c = std::min<int64_t>(4, row / wmin);
     if (bytes < ((size_t)8 << 20)) c = 1;   // small calls: latency, not bandwidth
     if (const char* e = getenv("DTC_HOST_CHUNKS")) c = atoi(e);
     return (int)std::max<int64_t>(1, std::min<int64_t>({c, 16, (N + 31) / 32}));   // widths: multiples of 32 columns
@@ -2189,7 +2193,7 @@ extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int6
         }
         h->stage_C_bytes = cbytes;
     }
-    const int nch = host_chunks(N, elt, bbytes + cbytes);
+    const int nch = host_chunks(h, N, elt, bbytes + cbytes);
     if (nch <= 1) {
         if (h->K > 0)
             DTC_CUDA(cudaMemcpy2DAsync(h->stage_B, N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice, s));
