@@ -495,7 +495,7 @@ static void free_format(dtc_format* h, cudaStream_t s) {
     dfree(h->vals, s); dfree(h->mask, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
     for (auto& e : h->hev) if (e) { cudaEventDestroy(e); e = nullptr; }
     for (auto& hs : h->hstream) if (hs) { cudaStreamDestroy(hs); hs = nullptr; }
-    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s); dfree(h->units_lpt, s);
+    dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s); dfree(h->units_lpt, s); dfree(h->ufirst, s);
 }
 
 struct BuildTemps {

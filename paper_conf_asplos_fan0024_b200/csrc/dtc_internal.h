@@ -64,6 +64,7 @@ struct dtc_format {
     int32_t* uctr = nullptr;
     int64_t uctr_len = 0;
     dtc::Unit* units_lpt = nullptr;   // units by size, descending (persistent launch)
+    int32_t* ufirst = nullptr;        // per-unit first-batch side records (one-CTA-per-unit pad launch)
     // GraphConv (dtc_graphconv): cuBLASLt workspace for the dense (A*H)*W step
     uint8_t* gemm_ws = nullptr;
     size_t gemm_ws_bytes = 0;

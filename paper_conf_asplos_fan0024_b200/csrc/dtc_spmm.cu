@@ -1156,6 +1156,10 @@ constexpr int pad_stages() {
 #define DTC_PAD_BATCH 16
 #endif
 constexpr int kPadBatch = DTC_PAD_BATCH;
+// per-unit side record for the first batch (default on; DTC_PAD_FIRST=0 disables): kPadBatch x 8 SparseAtoB ids
+// (-1 past the unit), TCOffset[bb], TCOffset[bb + min(kPadBatch, nb)], end of the first window, pad
+constexpr int kFirstRec = kPadBatch * 8 + 4;
+static_assert((kFirstRec * 4) % 16 == 0, "int4 loads of the side record");
 constexpr int kPadAValBytes = kPadBatch * 512 + 128;       // >= batch x 128 values x 4 B + 16, 128-aligned
 constexpr int kPadAIdsOff = kPadAValBytes + kPadBatch * 16;  // + one 16-byte mask per block
 constexpr int kPadASlot = kPadAIdsOff + kPadBatch * 32;      // + 8 SparseAtoB ids per block (hybrid LDG warps)
@@ -1214,7 +1218,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
            float* __restrict__ ws, int32_t* __restrict__ counters, int64_t npad,
            const int32_t* __restrict__ rowmap, int64_t* __restrict__ trace, const void* __restrict__ B,
-           int64_t ldb, int num_units, int32_t* __restrict__ uctr, int te, int lsur) {
+           int64_t ldb, int num_units, int32_t* __restrict__ uctr, int te, int lsur,
+           const int32_t* __restrict__ ufirst) {
     using Tr = Traits<DT>;
     constexpr int NJ1 = Tr::NJ, COLW1 = Tr::COLW, FW = Tr::FRAG_WORDS;
     constexpr int ELT = (int)sizeof(typename Tr::elt);
@@ -1325,8 +1330,24 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         q1 = bcast(q1);
         Unit u = q0 < num_units ? units[q0] : kNone;
         Unit un = q1 < num_units ? units[q1] : kNone;
-        int end0 = first_end(u), end0n = INT_MAX;
-        Raw rnext = load_raw(u, 0);
+        int end0, end0n = INT_MAX;
+        Raw rnext;
+        if (ufirst && q0 < num_units) {
+            // first unit of a one-CTA-per-unit launch: its first batch's SparseAtoB ids, TCOffset
+            // bounds and first-window end come from the unit's side record (indexed by blockIdx.x),
+            // so they load in parallel with the unit record instead of after it
+            const int32_t* fr = ufirst + (int64_t)q0 * kFirstRec;
+            rnext.mine = __ldg(reinterpret_cast<const int4*>(fr + jl * 8) + half);
+            rnext.e0 = rnext.e1 = 0;
+            if (lane == 0) {
+                rnext.e0 = __ldg(fr + kPadBatch * 8);
+                rnext.e1 = __ldg(fr + kPadBatch * 8 + 1);
+            }
+            end0 = __ldg(fr + kPadBatch * 8 + 2);
+        } else {
+            end0 = first_end(u);
+            rnext = load_raw(u, 0);
+        }
         int gi0 = 0, gc0 = 0;
         for (int ord = 0;; ++ord) {
         // publish unit ord to the consumers (index -1 = no more units)
@@ -1866,12 +1887,56 @@ static bool pad_persistent() {
 
 // Dual-engine gather (DTC_PAD_LSU=k): every k-th TC block of a CTA is gathered by the producer warp
 // with cp.async (LSU path) instead of TMA gather4; 0 = TMA only.
+#ifndef DTC_PAD_FIRST_DEFAULT
+#define DTC_PAD_FIRST_DEFAULT 1
+#endif
 #ifndef DTC_PAD_LSU_DEFAULT
 #define DTC_PAD_LSU_DEFAULT 0
 #endif
 static int pad_lsu_every() {   // read per launch (experiments flip it between calls)
     const char* e = getenv("DTC_PAD_LSU");
     return e ? std::max(0, atoi(e)) : DTC_PAD_LSU_DEFAULT;
+}
+
+static bool pad_first() {   // DTC_PAD_FIRST=0/1 (read per launch; experiments flip it between calls)
+    const char* e = getenv("DTC_PAD_FIRST");
+    return e ? atoi(e) > 0 : DTC_PAD_FIRST_DEFAULT;
+}
+
+__global__ void k_units_first(int64_t nu, const Unit* __restrict__ units, const int32_t* __restrict__ atob,
+                              const int32_t* __restrict__ tco, const int32_t* __restrict__ rwo,
+                              int32_t* __restrict__ out) {
+    for (int64_t q = blockIdx.x; q < nu; q += gridDim.x) {
+        const Unit u = units[q];
+        const int nb = u.be - u.bb;
+        int32_t* o = out + q * kFirstRec;
+        for (int t = threadIdx.x; t < kFirstRec; t += blockDim.x) {
+            int32_t v = 0;
+            if (t < kPadBatch * 8) {
+                const int i = t / 8;
+                v = i < nb ? atob[(int64_t)(u.bb + i) * 8 + (t % 8)] : -1;
+            } else if (t == kPadBatch * 8) {
+                v = nb > 0 ? tco[u.bb] : 0;
+            } else if (t == kPadBatch * 8 + 1) {
+                v = nb > 0 ? tco[u.bb + min(kPadBatch, nb)] : 0;
+            } else if (t == kPadBatch * 8 + 2) {
+                v = (u.split_id < 0 && u.wb < u.we) ? rwo[u.wb + 1] : INT_MAX;
+            }
+            o[t] = v;
+        }
+    }
+}
+
+static cudaError_t first_records(dtc_format* h, cudaStream_t s) {
+    if (h->ufirst || h->num_units == 0) return cudaSuccess;
+    int32_t* d = nullptr;
+    if (dalloc(&d, (size_t)h->num_units * kFirstRec, s) != DTC_OK) return cudaErrorMemoryAllocation;
+    k_units_first<<<(unsigned)std::min<int64_t>(h->num_units, 65535), 128, 0, s>>>(h->num_units, h->units, h->atob,
+                                                                                  h->tco, h->rwo, d);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { dfree(d, s); return e; }
+    h->ufirst = d;
+    return cudaSuccess;
 }
 
 // Unit order for the persistent launch: largest units first (stable; longest-processing-time
@@ -1931,12 +1996,18 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
         }
     }
     const Unit* units = (uctr && a.h->units_lpt) ? a.h->units_lpt : a.h->units;
+    const int32_t* ufirst = nullptr;
+    if (NL == 0 && gx == a.h->num_units && pad_first()) {
+        cudaError_t e = first_records(a.h, a.s);
+        if (e != cudaSuccess) return e;
+        ufirst = a.h->ufirst;
+    }
     dim3 grid((unsigned)gx, (unsigned)a.gy);
     k_spmm_pad<DT, SL, SEG, NL, VEC><<<grid, (SL * SEG / 2 + NL + 1) * 32, smem, a.s>>>(
         map, units, a.h->rwo, a.h->tco, reinterpret_cast<const uint4*>(a.h->mask), a.h->atob, a.h->vals, a.C,
         a.ldc, a.h->M, a.N, a.h->ws, a.h->counters, a.npad, a.h->rowmap,
         (g_trace && (int64_t)grid.x * grid.y <= g_trace_cap) ? g_trace : nullptr, a.B, a.ldb, (int)a.h->num_units,
-        uctr, a.te, pad_lsu_every());
+        uctr, a.te, pad_lsu_every(), ufirst);
     return cudaGetLastError();
 }
 

@@ -197,3 +197,24 @@ def test_persistent_many_column_groups(dtype, N):
         set_spmm_path("default")
     assert np.array_equal(C0, C1) and np.array_equal(C1, C2)
     check_tol(C1, M, K, rp, ci, v, B, dtype)
+
+
+@pytest.mark.parametrize("name,U,dtype,N", [("c2", 0, "tf32", 128), ("c2", 16, "tf32", 512), ("c1", 2, "tf32", 32),
+                                            ("c1", 2, "fp16", 256), ("c1", 0, "tf32", 33)])
+def test_first_batch_records_bit_identical(name, U, dtype, N, monkeypatch):
+    """DTC_PAD_FIRST: the CTA's first batch from the per-unit side record (ids, TCOffset bounds,
+    first-window end) computes exactly what the unit-record path computes, and matches O1."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U)
+    monkeypatch.setenv("DTC_PAD_FIRST", "0")
+    C0 = spmm(f, B)
+    monkeypatch.setenv("DTC_PAD_FIRST", "1")
+    C1 = spmm(f, B)
+    C2 = spmm(f, B)
+    assert np.array_equal(C0, C1) and np.array_equal(C1, C2)
+    check_tol(C1, cfg.M, cfg.K, rp, ci, v, B, dtype)
