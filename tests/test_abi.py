@@ -5,6 +5,7 @@ import ctypes
 import os
 import re
 import subprocess
+import sys
 
 import numpy as np
 import pytest
@@ -95,3 +96,15 @@ def test_default_spmm_kernels_do_not_spill():
             local = int(re.search(r"LOCAL:(\d+)", lines[i + 1]).group(1))
             assert stack == 0 and local == 0, (m.group(1)[:60], lines[i + 1])
     assert seen >= 6
+
+
+def test_missing_library_fails_loudly(tmp_path):
+    """No CPU fallback: with libdtc.so absent the binding raises on the first call into the path."""
+    code = ("import sys, paper_conf_asplos_fan0024_b200 as d\n"
+            "try:\n    d.lib()\nexcept ImportError as e:\n    print('raised', 'no CPU fallback' in str(e)); sys.exit(0)\n"
+            "sys.exit(3)\n")
+    env = dict(os.environ, DTC_LIBRARY=str(tmp_path / "libdtc.so"))
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], env=env, cwd=root, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr
+    assert "raised True" in r.stdout
