@@ -138,7 +138,8 @@ int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, float* C, in
  * the copy-in of chunk j+1 overlaps chunk j's kernel and copy-out on library-owned streams;
  * the result is bit-identical to one dtc_spmm over all N columns.  Chunks: up to 4, each >= 512 B
  * of a B row (>= 256 B when the format is smaller than B); DTC_HOST_CHUNKS=k overrides
- * (1 = unpipelined). */
+ * (1 = unpipelined).  When the format is larger than B (long kernels) and C_host is pinned and
+ * mapped, the kernel stores C straight into C_host (no copy-out); DTC_HOST_ZC=0/1 overrides. */
 int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                   int64_t ldc, void* stream);
 

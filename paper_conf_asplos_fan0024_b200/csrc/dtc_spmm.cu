@@ -2265,6 +2265,48 @@ extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int6
         h->stage_C_bytes = cbytes;
     }
     const int nch = host_chunks(h, N, elt, bbytes + cbytes);
+    // Zero-copy C: when C_host is pinned and mapped, the kernel stores C straight into host memory
+    // (posted PCIe writes spread over the kernel) and the copy-out disappears.  It pays when the
+    // kernel is long next to the copies (format larger than B: c3 e2e 12.1 -> 10.1 ms) and costs
+    // 1-5% otherwise (c2, c4, c5; profiles/r01_host_zc.txt).  DTC_HOST_ZC=0/1 overrides.
+    float* Czc = nullptr;
+    {
+        const double fmt_bytes = (double)h->nnz * (elt + 1) + 36.0 * (double)h->T + 4.0 * (double)h->W;
+        bool zc = fmt_bytes > (double)bbytes && bbytes + cbytes >= ((size_t)8 << 20);
+        if (const char* e = getenv("DTC_HOST_ZC")) zc = atoi(e) > 0;
+        cudaPointerAttributes at{};
+        if (zc && cudaPointerGetAttributes(&at, C_host) == cudaSuccess && at.type == cudaMemoryTypeHost &&
+            at.devicePointer)
+            Czc = reinterpret_cast<float*>(at.devicePointer);
+        cudaGetLastError();
+    }
+    if (Czc) {
+        for (auto& hs : h->hstream)
+            if (!hs) DTC_CUDA(cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking));
+        for (auto& e : h->hev)
+            if (!e) DTC_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        cudaStream_t sin = h->hstream[0];
+        DTC_CUDA(cudaEventRecord(h->hev[32], s));
+        DTC_CUDA(cudaStreamWaitEvent(sin, h->hev[32], 0));
+        const int64_t units32 = (N + 31) / 32;
+        int64_t c0 = 0;
+        uint8_t* sb = reinterpret_cast<uint8_t*>(h->stage_B);
+        for (int j = 0; j < nch; ++j) {
+            const int64_t u = units32 / nch + (j < units32 % nch ? 1 : 0);
+            const int64_t nc = std::min<int64_t>(N - c0, u * 32);
+            uint8_t* bj = sb + (size_t)h->K * c0 * elt;
+            if (h->K > 0)
+                DTC_CUDA(cudaMemcpy2DAsync(bj, nc * elt, reinterpret_cast<const uint8_t*>(B_host) + c0 * elt,
+                                           ldb * elt, nc * elt, h->K, cudaMemcpyHostToDevice, sin));
+            DTC_CUDA(cudaEventRecord(h->hev[j], sin));
+            DTC_CUDA(cudaStreamWaitEvent(s, h->hev[j], 0));
+            int rc = spmm_launch(h, bj, nc, nc, Czc + c0, ldc, s);
+            if (rc) return rc;
+            c0 += nc;
+        }
+        DTC_CUDA(cudaStreamSynchronize(s));
+        return DTC_OK;
+    }
     if (nch <= 1) {
         if (h->K > 0)
             DTC_CUDA(cudaMemcpy2DAsync(h->stage_B, N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice, s));

@@ -258,3 +258,27 @@ def test_host_api_column_chunks(chunks, dtype, N, monkeypatch):
     # a second call reuses the staging buffers, streams and events
     Ch2 = f.spmm_host(np.ascontiguousarray(B))
     assert np.array_equal(Ch, Ch2)
+
+
+@pytest.mark.parametrize("zc", ["0", "1"])
+@pytest.mark.parametrize("chunks", ["1", "2", "4"])
+def test_host_api_pinned_zero_copy(zc, chunks, monkeypatch):
+    """dtc_spmm_host with pinned torch buffers; DTC_HOST_ZC=1 stores C straight into the mapped
+    host buffer (no copy-out).  Same C as dtc_spmm, bit for bit, including a padded ldc."""
+    import torch
+    monkeypatch.setenv("DTC_HOST_ZC", zc)
+    monkeypatch.setenv("DTC_HOST_CHUNKS", chunks)
+    M, K, N = 4000, 3500, 128
+    rp, ci = datagen.random_csr(M, K, 0.01, 11)
+    v = datagen.uniform(N, 5, len(ci))
+    B = datagen.uniform(N, 6, K * N).reshape(K, N)
+    f = build(M, K, rp, ci, v)
+    Cd = spmm(f, B)
+    Bh = torch.from_numpy(B).pin_memory()
+    Ch = torch.full((M, N), float("nan"), dtype=torch.float32).pin_memory()
+    f.spmm_host(Bh, Ch)
+    assert np.array_equal(Ch.numpy(), Cd)
+    Cw = torch.full((M, N + 4), -7.0, dtype=torch.float32).pin_memory()   # ldc = N + 4
+    f.spmm_host(Bh, Cw[:, :N])
+    assert np.array_equal(Cw[:, :N].numpy(), Cd)
+    assert torch.all(Cw[:, N:] == -7.0)
