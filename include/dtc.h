@@ -137,42 +137,58 @@ int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, float* C, in
  * Calls of >= 8 MB are pipelined over column chunks (C(:, cols) depends only on B(:, cols)):
  * the copy-in of chunk j+1 overlaps chunk j's kernel and copy-out on library-owned streams;
  * the result is bit-identical to one dtc_spmm over all N columns.  Chunks: up to 4, each >= 512 B
- * of a B row (>= 256 B when the format is smaller than B); DTC_HOST_CHUNKS=k overrides
- * (1 = unpipelined).  When the format is larger than B (long kernels) and C_host is pinned and
- * mapped, the kernel stores C straight into C_host (no copy-out); DTC_HOST_ZC=0/1 overrides. */
+ * of a B row (>= 256 B when the format is smaller than B).  When the format is larger than B (long kernels) and C_host is pinned and
+ * mapped, the kernel stores C straight into C_host (no copy-out).  DTC_OPT_HOST_CHUNKS and
+ * DTC_OPT_HOST_ZERO_COPY override both choices; DTC_OPT_LAST_HOST_MODE reports them.  The caller
+ * guarantees B_host holds K rows of ldb elements of the handle's dtype and C_host M rows of ldc
+ * floats (the library cannot check host extents).  On error no copy is left running against the
+ * host buffers. */
 int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                   int64_t ldc, void* stream);
 
 /* Number of kernels dtc_spmm launches per call (for launch accounting). */
 int dtc_spmm_launches_per_call(void);
 
-/* Kernel variant used by dtc_spmm (ablations and the per-path parity tests).
- * All variants compute the same S1-S5 and pass the same parity bar:
- *   0 = library default, 1 = register gather with shared-memory A chunks (the paper's
- *   FetchSparse/SDB structure), 2 = TMA tile::gather4 B ring,
- *   3 = direct: each warp builds its A fragment from TCValues via the per-block
- *   occupancy mask (no shared memory, no CTA barrier), 4 = TMA gather4 of whole
- *   512-byte row slices into 528-byte padded smem rows (conflict-free fragment reads).
- * Process-wide, takes effect at the next dtc_spmm; the environment variable
- * DTC_SPMM_PATH=ldg|tma|dir|pad sets the initial value.  Returns the previous setting
- * (0 if it was the default), or DTC_ERR_INVALID for an unknown path. */
-int dtc_set_spmm_path(int path);
-
-/* Persistent launch of the padded-row path (path 4): on = 1 launches one wave of CTAs (resident
- * CTAs per SM x SMs) that walk the F4 units in a static stride, the B ring and A batches of a CTA
- * running across unit boundaries (no per-unit pipeline fill, no CTA launch per unit); on = 0
- * launches one CTA per unit.  Same arithmetic and results either way (bit-identical: every unit
- * is computed by one CTA in the same order).  Process-wide; DTC_PAD_PERS=0|1 sets the initial
- * value.  Returns the previous setting. */
-int dtc_set_pad_persistent(int on);
+/* Per-handle launch options (defaults are the measured best).  Options change how
+ * dtc_spmm / dtc_spmm_host run, never what they compute: every setting gives the same C within
+ * the north_star tolerance, and the padded-path options give bit-identical C (tested).
+ *   DTC_OPT_KERNEL         0 auto = TMA padded-row kernel (k_spmm_pad) where TMA can describe B
+ *                          (16-byte aligned base and row pitch), else the register-gather kernel
+ *                          (k_spmm_ldg, the paper's FetchSparse/VFetchDense structure);
+ *                          1 forces the register-gather kernel; 4 requests the padded kernel
+ *                          (it still falls back where TMA cannot describe B).
+ *   DTC_OPT_PERSISTENT     padded kernel: 1 = one wave of CTAs drawing F4 units from an atomic
+ *                          counter, largest first; 0 = one CTA per unit (default).
+ *   DTC_OPT_FIRST_RECORDS  padded kernel: 1 = per-unit side records of the first batch (default).
+ *   DTC_OPT_HOST_CHUNKS    dtc_spmm_host column chunks, 0 = auto, 1..16.
+ *   DTC_OPT_HOST_ZERO_COPY dtc_spmm_host stores C straight into pinned mapped C_host:
+ *                          -1 = auto (when the format is larger than B), 0 = off, 1 = on.
+ *   DTC_OPT_SLICE_BYTES    padded kernel row slice per gather4 op: 0 auto, 512 or 1024.
+ *   DTC_OPT_LAST_KERNEL    read-only: kernel the last dtc_spmm ran (1 register gather, 4 padded).
+ *   DTC_OPT_LAST_HOST_MODE read-only: last dtc_spmm_host: 2 * column chunks + (1 if C was stored
+ *                          zero-copy into host memory, i.e. no device-to-host copy).
+ * Not synchronised against concurrent calls on the same handle (like dtc_spmm itself).
+ * Errors: INVALID (null handle, unknown option, value out of range, read-only option). */
+typedef enum {
+    DTC_OPT_KERNEL = 1,
+    DTC_OPT_PERSISTENT = 2,
+    DTC_OPT_FIRST_RECORDS = 3,
+    DTC_OPT_HOST_CHUNKS = 4,
+    DTC_OPT_HOST_ZERO_COPY = 5,
+    DTC_OPT_SLICE_BYTES = 6,
+    DTC_OPT_LAST_KERNEL = 100,
+    DTC_OPT_LAST_HOST_MODE = 101
+} dtc_option_t;
+int dtc_format_set_option(dtc_handle_t h, int32_t option, int64_t value);
+int dtc_format_get_option(dtc_handle_t h, int32_t option, int64_t* value);
 
 /* Diagnostics (the paper's per-SM busy/idle methodology, Fig. 3 P:152-160 / Fig. 15):
- * while enabled, each CTA of the TMA-path kernel writes 8 int64 to dev_buf[cta*8 ..]:
- * {cta, smid, t_start, t_first_issue, t_first_data, t_consumer_done, num_tc_blocks,
- * t_producer_done}, times in ns of the %globaltimer.  dev_buf is a caller-owned device buffer of
- * capacity_ctas*8 int64; launches with more CTAs than capacity_ctas are not traced.
- * capacity_ctas = 0 disables.  Process-wide.  Errors: INVALID. */
-int dtc_set_trace(void* dev_buf, int64_t capacity_ctas);
+ * while enabled, each CTA of the padded kernel launched for handle h writes 8 int64 to
+ * dev_buf[cta*8 ..]: {cta, smid, t_start, t_first_issue, t_first_data, t_consumer_done,
+ * num_tc_blocks, t_producer_done}, times in ns of the %globaltimer.  dev_buf is a caller-owned
+ * device buffer of capacity_ctas*8 int64 that must outlive its use; launches with more CTAs than
+ * capacity_ctas are not traced.  capacity_ctas = 0 disables.  Errors: INVALID. */
+int dtc_format_set_trace(dtc_handle_t h, void* dev_buf, int64_t capacity_ctas);
 
 void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory */
 

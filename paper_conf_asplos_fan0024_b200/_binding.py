@@ -75,9 +75,9 @@ def lib():
             L.dtc_spmm.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_launches_per_call.argtypes = []
-            L.dtc_set_spmm_path.argtypes = [ctypes.c_int]
-            L.dtc_set_pad_persistent.argtypes = [ctypes.c_int]
-            L.dtc_set_trace.argtypes = [_vp, _i64]
+            L.dtc_format_set_option.argtypes = [_vp, _i32, _i64]
+            L.dtc_format_get_option.argtypes = [_vp, _i32, _vp]
+            L.dtc_format_set_trace.argtypes = [_vp, _vp, _i64]
             L.dtc_format_destroy.argtypes = [_vp]
             L.dtc_format_destroy.restype = None
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
@@ -128,32 +128,10 @@ def launches_per_call() -> int:
     return int(lib().dtc_spmm_launches_per_call())
 
 
-SPMM_PATHS = {"default": 0, "ldg": 1, "tma": 2, "dir": 3, "pad": 4}
-
-
-def set_trace(buf=None) -> None:
-    """Enable (CUDA int64 tensor of shape [ctas, 8]) or disable (None) the per-CTA timeline."""
-    if buf is None:
-        _check(lib().dtc_set_trace(None, 0), "dtc_set_trace")
-        return
-    import torch
-    if buf.dtype != torch.int64 or not buf.is_cuda or buf.dim() != 2 or buf.shape[1] != 8:
-        raise TypeError("trace buffer must be a CUDA int64 tensor [ctas, 8]")
-    _check(lib().dtc_set_trace(ctypes.c_void_p(buf.data_ptr()), buf.shape[0]), "dtc_set_trace")
-
-
-def set_pad_persistent(on: bool) -> bool:
-    """Persistent (one-wave) launch of the padded-row SpMM path (dtc_set_pad_persistent)."""
-    return bool(lib().dtc_set_pad_persistent(1 if on else 0))
-
-
-def set_spmm_path(path) -> int:
-    """Select the dtc_spmm kernel variant (include/dtc.h dtc_set_spmm_path); returns the previous one."""
-    code = SPMM_PATHS[path] if isinstance(path, str) else int(path)
-    st = int(lib().dtc_set_spmm_path(code))
-    if st < 0:
-        _check(st, "dtc_set_spmm_path")
-    return st
+# per-handle launch options (include/dtc.h dtc_option_t)
+OPTIONS = {"kernel": 1, "persistent": 2, "first_records": 3, "host_chunks": 4, "host_zero_copy": 5,
+           "slice_bytes": 6, "last_kernel": 100, "last_host_mode": 101}
+KERNELS = {"auto": 0, "ldg": 1, "pad": 4}
 
 
 def _dtype_code(dtype) -> int:
@@ -190,7 +168,7 @@ def _make_csr(rowptr, colidx, vals, M, K, dtype) -> _Csr:
 class Format:
     """An ME-TCF handle (library-owned device memory)."""
 
-    def __init__(self, handle: int, keep=()):
+    def __init__(self, handle: int, keep=(), device: int = 0):
         self._h = ctypes.c_void_p(handle)
         self._keep = keep
         v = self.query()
@@ -199,6 +177,8 @@ class Format:
         self.num_units, self.num_split_windows = v.num_units, v.num_split_windows
         self.unit_blocks = v.unit_blocks
         self.dtype = "fp16" if v.dtype == DTC_FP16 else "tf32"
+        self.device = device
+        self._trace = None
 
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
@@ -215,7 +195,7 @@ class Format:
         opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
-        return cls(h.value)
+        return cls(h.value, device=rowptr.device.index or 0)
 
     @property
     def handle(self):
@@ -248,19 +228,54 @@ class Format:
         out["num_tc_blocks"] = T
         return out
 
+    def set_option(self, name, value) -> None:
+        """Per-handle launch option (dtc_format_set_option): kernel ("auto" | "ldg" | "pad"),
+        persistent, first_records, host_chunks, host_zero_copy, slice_bytes."""
+        if name == "kernel" and isinstance(value, str):
+            value = KERNELS[value]
+        _check(lib().dtc_format_set_option(self._h, OPTIONS[name], int(value)), "dtc_format_set_option")
+
+    def get_option(self, name) -> int:
+        v = _i64()
+        _check(lib().dtc_format_get_option(self._h, OPTIONS[name], ctypes.byref(v)), "dtc_format_get_option")
+        return int(v.value)
+
+    def set_trace(self, buf=None) -> None:
+        """Enable (CUDA int64 tensor of shape [ctas, 8]) or disable (None) the per-CTA timeline."""
+        if buf is None:
+            _check(lib().dtc_format_set_trace(self._h, None, 0), "dtc_format_set_trace")
+            self._trace = None
+            return
+        import torch
+        if buf.dtype != torch.int64 or not buf.is_cuda or buf.dim() != 2 or buf.shape[1] != 8 or not buf.is_contiguous():
+            raise TypeError("trace buffer must be a contiguous CUDA int64 tensor [ctas, 8]")
+        _check(lib().dtc_format_set_trace(self._h, ctypes.c_void_p(buf.data_ptr()), buf.shape[0]),
+               "dtc_format_set_trace")
+        self._trace = buf   # keep it alive while the library may write to it
+
+    def _want(self):
+        import torch
+        return torch.float16 if self.dtype == "fp16" else torch.float32
+
     def spmm(self, B, C=None, stream=None):
         """C := A @ B on the GPU (B: CUDA tensor K x N of the handle dtype, row stride ldb)."""
         import torch
-        if B.dim() != 2 or not B.is_cuda or B.stride(1) != 1:
+        if not isinstance(B, torch.Tensor) or B.dim() != 2 or not B.is_cuda or B.stride(1) != 1:
             raise TypeError("B must be a 2-D CUDA tensor with unit column stride")
-        want = torch.float16 if self.dtype == "fp16" else torch.float32
-        if B.dtype != want:
-            raise TypeError(f"B must be {want}")
+        if B.dtype != self._want():
+            raise TypeError(f"B must be {self._want()}")
+        if B.shape[0] != self.K:
+            raise ValueError(f"B must have K = {self.K} rows, got {B.shape[0]}")
+        if B.device.index != self.device:
+            raise ValueError(f"B is on {B.device}, the handle on cuda:{self.device}")
         N = B.shape[1]
         if C is None:
             C = torch.empty((self.M, N), dtype=torch.float32, device=B.device)
-        if C.dtype != torch.float32 or C.stride(1) != 1 or C.shape[0] != self.M or C.shape[1] != N:
+        if (not isinstance(C, torch.Tensor) or C.dtype != torch.float32 or not C.is_cuda or C.dim() != 2
+                or C.stride(1) != 1 or C.shape[0] != self.M or C.shape[1] != N):
             raise TypeError("C must be a float32 (M x N) CUDA tensor with unit column stride")
+        if C.device.index != self.device:
+            raise ValueError(f"C is on {C.device}, the handle on cuda:{self.device}")
         _check(lib().dtc_spmm(self._h, _dptr(B), N, B.stride(0), _dptr(C), C.stride(0), _stream_ptr(stream)),
                "dtc_spmm")
         return C
@@ -270,9 +285,11 @@ class Format:
         H: CUDA K x F_in (handle dtype), W: CUDA fp32 F_in x F_out, bias fp32 F_out or None.
         Returns (Y, AH); all tensors contiguous row-major."""
         import torch
-        want = torch.float16 if self.dtype == "fp16" else torch.float32
+        want = self._want()
         if H.dtype != want or not H.is_cuda or not H.is_contiguous() or H.dim() != 2:
             raise TypeError(f"H must be a contiguous 2-D CUDA {want} tensor")
+        if H.shape[0] != self.K:
+            raise ValueError(f"H must have K = {self.K} rows, got {H.shape[0]}")
         F_in, F_out = H.shape[1], W.shape[1]
         if W.dtype != torch.float32 or not W.is_contiguous() or W.shape[0] != F_in:
             raise TypeError("W must be a contiguous fp32 (F_in x F_out) tensor")
@@ -293,11 +310,19 @@ class Format:
         _check(lib().dtc_spmm(self._h, B_ptr, N, ldb, C_ptr, ldc, _stream_ptr(stream)), "dtc_spmm")
 
     def spmm_host(self, B_host, C_host=None, stream=None):
-        """End-to-end C = A @ B with HOST buffers (numpy or pinned torch CPU tensors)."""
-        bp, N, ldb = _host_ptr(B_host)
+        """End-to-end C = A @ B with HOST buffers (numpy or pinned torch CPU tensors).  The library
+        cannot see host extents, so B (K x N, handle dtype) and C (M x N, float32) are checked here."""
+        bp, (K, N), ldb, bdt = _host_ptr(B_host, "B_host")
+        want = np.float16 if self.dtype == "fp16" else np.float32
+        if bdt != np.dtype(want):
+            raise TypeError(f"B_host must be {np.dtype(want)}, got {bdt}")
+        if K != self.K:
+            raise ValueError(f"B_host must have K = {self.K} rows, got {K}")
         if C_host is None:
             C_host = np.empty((self.M, N), dtype=np.float32)
-        cp, _, ldc = _host_ptr(C_host)
+        cp, (M, Nc), ldc, cdt = _host_ptr(C_host, "C_host")
+        if cdt != np.dtype(np.float32) or (M, Nc) != (self.M, N):
+            raise TypeError(f"C_host must be float32 of shape ({self.M}, {N}), got {cdt} {(M, Nc)}")
         _check(lib().dtc_spmm_host(self._h, bp, N, ldb, cp, ldc, _stream_ptr(stream)), "dtc_spmm_host")
         return C_host
 
@@ -313,13 +338,31 @@ class Format:
             pass
 
 
-def _host_ptr(a):
+def _host_ptr(a, name):
+    """(pointer, shape, row stride in elements, numpy dtype) of a 2-D host buffer with unit column stride."""
     if isinstance(a, np.ndarray):
-        assert a.ndim == 2 and a.strides[1] == a.itemsize
-        return a.ctypes.data, a.shape[1], a.strides[0] // a.itemsize
-    # torch CPU tensor
-    assert a.dim() == 2 and a.stride(1) == 1 and not a.is_cuda
-    return a.data_ptr(), a.shape[1], a.stride(0)
+        if a.ndim != 2 or a.strides[1] != a.itemsize or a.strides[0] % a.itemsize or a.strides[0] < 0:
+            raise TypeError(f"{name} must be a 2-D array with unit column stride")
+        return a.ctypes.data, a.shape, a.strides[0] // a.itemsize, a.dtype
+    import torch
+    if not isinstance(a, torch.Tensor) or a.is_cuda or a.dim() != 2 or a.stride(1) != 1:
+        raise TypeError(f"{name} must be a 2-D host array/tensor with unit column stride")
+    dt = {torch.float32: np.dtype(np.float32), torch.float16: np.dtype(np.float16)}.get(a.dtype, None)
+    if dt is None:
+        raise TypeError(f"{name} has unsupported dtype {a.dtype}")
+    return a.data_ptr(), tuple(a.shape), a.stride(0), dt
+
+
+def _dense(t, name, shape, dtype):
+    """Raise unless t is a contiguous 2-D CUDA tensor of `dtype` whose shape matches (None = any)."""
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dim() != 2 or not t.is_contiguous():
+        raise TypeError(f"{name} must be a contiguous 2-D CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    for got, want in zip(t.shape, shape):
+        if want is not None and got != want:
+            raise ValueError(f"{name} must have shape {shape}, got {tuple(t.shape)}")
 
 
 def partition_windows(rwo, world: int) -> np.ndarray:
@@ -379,16 +422,26 @@ class Dist:
         self.row_begin, self.row_end = rb.value, re_.value
         self._local = loc
 
+    def _want(self):
+        import torch
+        return torch.float16 if self.dtype == "fp16" else torch.float32
+
     def local_spmm(self, B, C_local, stream=None):
         """This rank's rows only, B already resident (no collective): C_local = A[rows] @ B."""
+        import torch
+        _dense(B, "B", (self.K, None), self._want())
         N = B.shape[1]
-        assert B.is_contiguous() and C_local.is_contiguous() and C_local.shape[0] >= self.row_end - self.row_begin
+        _dense(C_local, "C_local", (max(self.row_end - self.row_begin, 1), N), torch.float32)
         _check(lib().dtc_spmm(self._local, _dptr(B), N, N, _dptr(C_local), N, _stream_ptr(stream)), "dtc_spmm")
         return C_local
 
     def spmm(self, B, C, root: int = 0, gather_c: bool = True, stream=None):
+        """dtc_spmm_dist: B (K x N, valid on root) is broadcast; C is M x N (gather_c) or this rank's rows."""
+        import torch
+        _dense(B, "B", (self.K, None), self._want())
         N = B.shape[1]
-        assert B.is_contiguous() and C.is_contiguous()
+        rows = self.M if gather_c else max(self.row_end - self.row_begin, 1)
+        _dense(C, "C", (rows, N), torch.float32)
         _check(lib().dtc_spmm_dist(self._h, _dptr(B), root, N, _dptr(C), int(gather_c), _stream_ptr(stream)),
                "dtc_spmm_dist")
         return C

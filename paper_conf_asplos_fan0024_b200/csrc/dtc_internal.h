@@ -23,6 +23,16 @@ struct Unit {
 };
 static_assert(sizeof(Unit) == 32, "unit record is 8 x int32");
 
+// Per-handle launch options (dtc_format_set_option; include/dtc.h DTC_OPT_*).
+struct Options {
+    int32_t kernel = 0;          // 0 auto, 1 register gather, 4 TMA padded rows
+    int32_t persistent = 0;      // padded path: one wave of CTAs drawing units
+    int32_t first_records = 1;   // padded path: per-unit first-batch side records
+    int32_t host_chunks = 0;     // dtc_spmm_host column chunks, 0 = auto
+    int32_t host_zc = -1;        // dtc_spmm_host zero-copy C: -1 auto, 0 off, 1 on
+    int32_t slice_bytes = 0;     // padded path: 0 auto, 512 or 1024
+};
+
 }  // namespace dtc
 
 struct dtc_format {
@@ -60,6 +70,12 @@ struct dtc_format {
     cudaEvent_t hev[2 * 16 + 1] = {};
     // optional row map (row of the condensed matrix -> row of C), from dtc_build_opts_t.row_perm
     int32_t* rowmap = nullptr;
+    // launch options and diagnostics
+    dtc::Options opt;
+    int64_t* trace = nullptr;         // per-CTA timeline buffer (dtc_format_set_trace), caller-owned
+    int64_t trace_cap = 0;
+    int32_t last_kernel = 0;          // kernel of the last dtc_spmm (1 register gather, 4 padded TMA)
+    int64_t last_host_mode = 0;       // last dtc_spmm_host: 2 * chunks + zero-copy C
     // persistent padded-row launch: dynamic unit counters, 2 per column group (self-resetting)
     int32_t* uctr = nullptr;
     int64_t uctr_len = 0;

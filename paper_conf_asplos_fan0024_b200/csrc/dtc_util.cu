@@ -2,6 +2,7 @@
 // the format builder (F2, F3, F4).
 #include <cstdarg>
 #include <cstring>
+#include <mutex>
 
 #include "dtc_internal.h"
 
@@ -24,9 +25,11 @@ int cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
 
 cudaMemPool_t lib_pool() {
     static cudaMemPool_t pools[64] = {};
+    static std::mutex mu;
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
+    std::lock_guard<std::mutex> lock(mu);
     if (!pools[dev]) {
         cudaMemPoolProps props = {};
         props.allocType = cudaMemAllocationTypePinned;

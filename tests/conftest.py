@@ -28,3 +28,20 @@ def pytest_collection_modifyitems(config, items):
     for it in items:
         if "gpu" in it.keywords:
             it.add_marker(skip)
+
+
+_PARITY = {}
+
+
+@pytest.fixture(scope="session")
+def parity_report():
+    """name -> (worst err/limit, elements compared) of the full-size parity tests (printed at the end)."""
+    return _PARITY
+
+
+def pytest_terminal_summary(terminalreporter, exitstatus, config):
+    if not _PARITY:
+        return
+    terminalreporter.write_sep("-", "full-size parity vs oracle O1 (every element compared)")
+    for k, (worst, n) in sorted(_PARITY.items()):
+        terminalreporter.write_line(f"{k:32s} {n:>13,d} elements  worst err/limit {worst:.4f}")

@@ -85,8 +85,7 @@ def test_config_bit_exact(name):
     f = build(cfg.M, cfg.K, rp, ci, v, dtype=cfg.dtype)
     got = f.export()
     assert_format_equal(got, oracle.condense(cfg.M, rp, ci, v))
-    if cfg.M < 300000:
-        check_units(got, cfg.M)
+    check_units(got, cfg.M)
 
 
 def test_invalid_inputs():

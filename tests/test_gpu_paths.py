@@ -1,9 +1,10 @@
-"""Every dtc_spmm kernel variant (dtc_set_spmm_path: ldg / tma / dir / pad) against oracle O1.
+"""Every dtc_spmm launch variant (per-handle options, include/dtc.h DTC_OPT_*) against oracle O1.
 
 The library default is covered by test_gpu_spmm.py at every config; this module runs the
 same parity bar (tolerance of BASELINE.json north_star, bit-exact for the exact-arithmetic
-pins P2/P3/P9) on each variant, so an ablation number in profiles/ is never a number of an
-incorrect kernel.
+pins P2/P3/P9) on each variant -- the register-gather fallback kernel, the padded TMA kernel
+one CTA per unit, persistent, without first-batch records, and with 512-byte slices forced --
+so an ablation number in profiles/ is never a number of an incorrect kernel.
 """
 import numpy as np
 import pytest
@@ -12,28 +13,27 @@ import datagen
 import oracle
 from datagen import configs
 
-from gpu_util import build, dev, spmm, check_tol
+from gpu_util import build as _build, dev, spmm, check_tol
 
 pytestmark = pytest.mark.gpu
 
-PATHS = ["ldg", "tma", "dir", "pad", "hyb", "pers", "pershyb", "lsu2", "lsu3", "perslsu3"]
+VARIANTS = {
+    "ldg": {"kernel": "ldg"},
+    "pad": {"kernel": "pad"},
+    "pers": {"kernel": "pad", "persistent": 1},
+    "nofirst": {"kernel": "pad", "first_records": 0},
+    "slice512": {"kernel": "pad", "slice_bytes": 512},
+}
 
 
-@pytest.fixture(params=PATHS)
-def path(request, monkeypatch):
-    """hyb = the TMA path with half of every CTA's columns gathered by LSU warps (DTC_PAD_HYB);
-    pers* = the padded-row path launched persistently (one wave walking the units)."""
-    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
-    p = request.param
-    if p.endswith("hyb"):
-        monkeypatch.setenv("DTC_PAD_HYB", "1")
-    if "lsu" in p:   # dual-engine gather: every k-th block by cp.async
-        monkeypatch.setenv("DTC_PAD_LSU", p[-1])
-    prev = set_pad_persistent(p.startswith("pers"))
-    set_spmm_path("pad" if (p in ("hyb", "pers", "pershyb") or "lsu" in p) else p)
-    yield p
-    set_spmm_path("default")
-    set_pad_persistent(prev)
+@pytest.fixture(params=list(VARIANTS))
+def path(request):
+    return request.param
+
+
+def build(*a, path=None, **kw):
+    f = _build(*a, options=VARIANTS[path] if path else None, **kw)
+    return f
 
 
 @pytest.mark.parametrize("dtype", ["tf32", "fp16"])
@@ -45,8 +45,12 @@ def test_random_tolerance(path, dtype, N):
     B = datagen.uniform(N, 2, K * N).reshape(K, N)
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
-    f = build(M, K, rp, ci, v, dtype=dtype)
+    f = build(M, K, rp, ci, v, dtype=dtype, path=path)
     check_tol(spmm(f, B), M, K, rp, ci, v, B, dtype)
+    # the variant really ran: TMA needs whole 4-byte elements per row, else the register gather
+    elt = 2 if dtype == "fp16" else 4
+    want = 1 if path == "ldg" or (N * elt) % 4 else 4
+    assert f.get_option("last_kernel") == want
 
 
 @pytest.mark.parametrize("dtype", ["tf32", "fp16"])
@@ -59,7 +63,7 @@ def test_p2_integer_bit_exact(path, name, N, U, dtype):
     B = datagen.integers(cfg.seed_b, 6, cfg.K * N).reshape(cfg.K, N)
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
-    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U, path=path)
     C = spmm(f, B)
     assert np.array_equal(C, spmm(f, B))
     Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v.astype(np.float32), B.astype(np.float32))
@@ -77,7 +81,7 @@ def test_p9_dense_blocks_exact(path, dtype):
     B = datagen.integers(9, 2, K * N).reshape(K, N)
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
-    f = build(M, K, rp, ci, v, dtype=dtype)
+    f = build(M, K, rp, ci, v, dtype=dtype, path=path)
     C = spmm(f, B)
     ref = v.astype(np.float64).reshape(M, K) @ B.astype(np.float64)
     assert np.array_equal(C.astype(np.float64), ref)
@@ -91,7 +95,7 @@ def test_p3_identity_and_empty_windows(path):
     keep[100:180] = False                                              # 5 empty windows
     rp = np.concatenate([[0], np.cumsum(keep)]).astype(np.int32)
     ci = np.nonzero(keep)[0].astype(np.int32)
-    f = build(M, M, rp, ci, np.ones(len(ci), np.float32))
+    f = build(M, M, rp, ci, np.ones(len(ci), np.float32), path=path)
     ref = Bt * keep[:, None]
     assert np.array_equal(spmm(f, Bt), ref)
 
@@ -105,7 +109,7 @@ def test_strided_misaligned(path, dtype):
     Bf = datagen.uniform(7, 2, K * 50).reshape(K, 50)
     if dtype == "fp16":
         v, Bf = v.astype(np.float16), Bf.astype(np.float16)
-    f = build(M, K, rp, ci, v, dtype=dtype)
+    f = build(M, K, rp, ci, v, dtype=dtype, path=path)
     Bd = dev(Bf)[:, 1:1 + N]
     Cbig = torch.full((M, 41), float("nan"), device="cuda")
     C = Cbig[:, 2:2 + N]
@@ -122,7 +126,7 @@ def test_row_perm_original_order(path):
     N = 64
     B = datagen.integers(cfg.seed_b, 6, cfg.K * N).reshape(cfg.K, N)
     perm = np.random.default_rng(3).permutation(cfg.M).astype(np.int32)
-    f = build(cfg.M, cfg.K, rp, ci, v, row_perm=dev(perm))
+    f = build(cfg.M, cfg.K, rp, ci, v, row_perm=dev(perm), path=path)
     Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v, B)
     assert np.array_equal(spmm(f, B).astype(np.float64), Cr)
 
@@ -130,22 +134,14 @@ def test_row_perm_original_order(path):
 @pytest.mark.parametrize("name,U", [("c2", 0), ("c2", 16), ("c1", 2)])
 def test_persistent_bit_identical(name, U):
     """Persistent and one-CTA-per-unit launches compute every unit in the same order."""
-    import torch
-    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
     cfg = configs.get(name)
     rp, ci = configs.make_pattern(cfg)
     v = configs.make_values(cfg, len(ci))
     B = configs.make_B(cfg, cfg.N)
-    f = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U)
-    set_spmm_path("pad")
-    try:
-        prev = set_pad_persistent(False)
-        C0 = spmm(f, B)
-        set_pad_persistent(True)
-        C1 = spmm(f, B)
-        set_pad_persistent(prev)
-    finally:
-        set_spmm_path("default")
+    f = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U, path="pad")
+    C0 = spmm(f, B)
+    f.set_option("persistent", 1)
+    C1 = spmm(f, B)
     assert np.array_equal(C0, C1)
 
 
@@ -177,33 +173,26 @@ def test_unit_order_split_first(name, U):
 def test_persistent_many_column_groups(dtype, N):
     """Wide B (several CTA column groups, each with its own dynamic unit counter), split windows:
     persistent == one-CTA-per-unit bit for bit, and within tolerance of the oracle."""
-    from paper_conf_asplos_fan0024_b200 import set_spmm_path, set_pad_persistent
     M, K = 600, 500
     rp, ci = datagen.random_csr(M, K, 0.08, N)
     v = datagen.uniform(N, 1, len(ci))
     B = datagen.uniform(N, 2, K * N).reshape(K, N)
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
-    f = build(M, K, rp, ci, v, dtype=dtype, unit_blocks=4)
-    set_spmm_path("pad")
-    try:
-        prev = set_pad_persistent(False)
-        C0 = spmm(f, B)
-        set_pad_persistent(True)
-        C1 = spmm(f, B)
-        C2 = spmm(f, B)       # counters reset by the previous launch
-        set_pad_persistent(prev)
-    finally:
-        set_spmm_path("default")
+    f = build(M, K, rp, ci, v, dtype=dtype, unit_blocks=4, path="pad")
+    C0 = spmm(f, B)
+    f.set_option("persistent", 1)
+    C1 = spmm(f, B)
+    C2 = spmm(f, B)       # counters reset by the previous launch
     assert np.array_equal(C0, C1) and np.array_equal(C1, C2)
     check_tol(C1, M, K, rp, ci, v, B, dtype)
 
 
 @pytest.mark.parametrize("name,U,dtype,N", [("c2", 0, "tf32", 128), ("c2", 16, "tf32", 512), ("c1", 2, "tf32", 32),
                                             ("c1", 2, "fp16", 256), ("c1", 0, "tf32", 33)])
-def test_first_batch_records_bit_identical(name, U, dtype, N, monkeypatch):
-    """DTC_PAD_FIRST: the CTA's first batch from the per-unit side record (ids, TCOffset bounds,
-    first-window end) computes exactly what the unit-record path computes, and matches O1."""
+def test_first_batch_records_bit_identical(name, U, dtype, N):
+    """DTC_OPT_FIRST_RECORDS: the CTA's first batch from the per-unit side record (ids, TCOffset
+    bounds, first-window end) computes exactly what the unit-record path computes, and matches O1."""
     cfg = configs.get(name)
     rp, ci = configs.make_pattern(cfg)
     v = configs.make_values(cfg, len(ci))
@@ -211,10 +200,47 @@ def test_first_batch_records_bit_identical(name, U, dtype, N, monkeypatch):
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
     f = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, unit_blocks=U)
-    monkeypatch.setenv("DTC_PAD_FIRST", "0")
+    f.set_option("first_records", 0)
     C0 = spmm(f, B)
-    monkeypatch.setenv("DTC_PAD_FIRST", "1")
+    f.set_option("first_records", 1)
     C1 = spmm(f, B)
     C2 = spmm(f, B)
     assert np.array_equal(C0, C1) and np.array_equal(C1, C2)
     check_tol(C1, cfg.M, cfg.K, rp, ci, v, B, dtype)
+
+
+@pytest.mark.parametrize("U", [0, 1, 3])
+@pytest.mark.parametrize("name,N", [("c1", 64), ("c1", 256), ("c2", 128)])
+def test_fp16_block_pairs_exact(name, N, U):
+    """FP16 m16n8k16 over pairs of TC blocks of one window (odd tails and unit/split boundaries take
+    m16n8k8): integer inputs are exact either way, so C must equal O1 bit for bit, and the padded
+    kernel must equal the register-gather kernel (k8 per block) bit for bit."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = datagen.integers(cfg.seed_a, 7, len(ci)).astype(np.float16)
+    B = datagen.integers(cfg.seed_b, 8, cfg.K * N).reshape(cfg.K, N).astype(np.float16)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype="fp16", unit_blocks=U)
+    C = spmm(f, B)
+    assert f.get_option("last_kernel") == 4
+    Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, v.astype(np.float32), B.astype(np.float32))
+    assert np.array_equal(C.astype(np.float64), Cr)
+    f.set_option("kernel", "ldg")
+    assert np.array_equal(spmm(f, B), C)
+
+
+def test_options_roundtrip_and_errors():
+    from paper_conf_asplos_fan0024_b200 import DtcError
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    f = build(cfg.M, cfg.K, rp, ci, v)
+    defaults = {"kernel": 0, "persistent": 0, "first_records": 1, "host_chunks": 0, "host_zero_copy": -1,
+                "slice_bytes": 0}
+    for k, x in defaults.items():
+        assert f.get_option(k) == x
+    for k, bad in (("kernel", 2), ("persistent", 5), ("host_chunks", 17), ("host_zero_copy", 2),
+                   ("slice_bytes", 256), ("last_kernel", 1)):
+        with pytest.raises(DtcError):
+            f.set_option(k, bad)
+    f.set_option("host_chunks", 3)
+    assert f.get_option("host_chunks") == 3

@@ -6,15 +6,14 @@ import numpy as np
 import torch
 import datagen
 from datagen import configs
-from paper_conf_asplos_fan0024_b200 import Format, set_spmm_path
+from paper_conf_asplos_fan0024_b200 import Format
 
 cfg = configs.get("c1")
 rp, ci = configs.make_pattern(cfg)
-for path in ("default", "ldg", "dir"):
-  set_spmm_path(path)
+for path in ("auto", "ldg", "pers"):
   for dtype in ("tf32", "fp16"):
     v = configs.make_values(cfg, len(ci))
-    for N in ((32, 37, 128, 256, 512) if path == "default" else (37, 128)):
+    for N in ((32, 37, 128, 256, 512) if path == "auto" else (37, 128)):
         B = datagen.uniform(1, 2, cfg.K * N).reshape(cfg.K, N)
         if dtype == "fp16":
             v, B = v.astype(np.float16), B.astype(np.float16)
@@ -22,6 +21,8 @@ for path in ("default", "ldg", "dir"):
             f = Format.build(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(),
                              torch.from_numpy(v if dtype == "fp16" else v.astype(np.float32)).cuda(),
                              cfg.M, cfg.K, dtype=dtype, unit_blocks=U)
+            f.set_option("kernel", "ldg" if path == "ldg" else "auto")
+            f.set_option("persistent", 1 if path == "pers" else 0)
             C = f.spmm(torch.from_numpy(B).cuda())
             torch.cuda.synchronize()
             f.close()

@@ -1,4 +1,4 @@
-"""Per-CTA timeline of the TMA-path SpMM kernel (dtc_set_trace) -- diagnostics, not product code.
+"""Per-CTA timeline of the TMA-path SpMM kernel (dtc_format_set_trace) -- diagnostics, not product code.
 
 The paper's per-SM busy/idle method (Fig. 3; Fig. 15) on B200:
     python tools/trace_cta.py c2 [--unit-blocks U] [--out gpurun_out/trace_c2.npz]
@@ -20,6 +20,7 @@ def main():
     ap.add_argument("config")
     ap.add_argument("--unit-blocks", type=int, default=0)
     ap.add_argument("--out", default="")
+    ap.add_argument("--persistent", type=int, default=0)
     a = ap.parse_args()
     import torch
     from datagen import configs
@@ -31,6 +32,7 @@ def main():
     B = configs.make_B(cfg, N)
     f = dtc.Format.build(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), torch.from_numpy(v).cuda(),
                          cfg.M, cfg.K, dtype=cfg.dtype, unit_blocks=a.unit_blocks)
+    f.set_option("persistent", a.persistent)
     Bd = torch.from_numpy(B).cuda()
     C = torch.empty((cfg.M, N), device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -40,10 +42,10 @@ def main():
         f.spmm(Bd, C)
     flush.zero_()
     torch.cuda.synchronize()
-    dtc.set_trace(tr)
+    f.set_trace(tr)
     f.spmm(Bd, C)
     torch.cuda.synchronize()
-    dtc.set_trace(None)
+    f.set_trace(None)
     t = tr.cpu().numpy()
     t = t[t[:, 2] > 0]
     t0 = t[:, 2].min()
