@@ -66,6 +66,8 @@ def parse_args():
     p.add_argument("--unit-blocks", type=int, default=0)
     p.add_argument("--guided", type=int, default=0, help="F4 guided tail (1 on, -1 off, 0 auto)")
     p.add_argument("--persistent", type=int, default=0, help="DTC_OPT_PERSISTENT for the timed launches")
+    p.add_argument("--selector", type=int, default=0,
+                   help="F4 cut by the B200 Selector's plan for this N (NEXT-4, dtc_selector_plan): 1 on, 0 fixed rule")
     p.add_argument("--ncu", default="auto", choices=["auto", "off"],
                    help="capture DRAM traffic of one launch per leg under ncu (subprocess)")
     p.add_argument("--no-cusparse", action="store_true")
@@ -243,7 +245,7 @@ def ncu_traffic(legs, cache_dir, timeout_s=600):
         launches.setdefault(int(d["ID"]), {})[d["Metric Name"]] = (float(d["Metric Value"].replace(",", "")),
                                                                    d["Metric Unit"])
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12, "nsecond": 1e-9, "usecond": 1e-6,
-             "msecond": 1e-3, "second": 1.0}
+             "msecond": 1e-3, "second": 1.0, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1.0}
     out = {}
     ids = sorted(launches)
     if len(ids) != len(legs):
@@ -253,7 +255,8 @@ def ncu_traffic(legs, cache_dir, timeout_s=600):
         g = lambda k: m[k][0] * scale.get(m[k][1], 1.0) if k in m else None  # noqa: E731
         rd, wr = g("dram__bytes_read.sum"), g("dram__bytes_write.sum")
         out[f"{name}:{N}"] = {"dram_bytes": int(rd + wr) if rd is not None and wr is not None else None,
-                              "kernel_s": g("gpu__time_duration.sum"), "l2_bytes": g("lts__t_bytes.sum")}
+                              "kernel_s": g("gpu__time_duration.sum"), "l2_bytes": g("lts__t_bytes.sum"),
+                              "time_unit": m.get("gpu__time_duration.sum", (0, "?"))[1]}
     return out
 
 
@@ -345,7 +348,7 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
         torch.cuda.synchronize()
         tb0 = time.perf_counter()
         fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks,
-                               guided=args.guided)
+                               guided=args.guided, n_hint=N, selector=args.selector)
         torch.cuda.synchronize()
         build_ms_runs.append((time.perf_counter() - tb0) * 1e3)
     fmt.set_option("persistent", args.persistent)
@@ -368,7 +371,9 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
     T = fmt.num_tc_blocks
     leg.update({"num_tc_blocks": T, "mean_nnz_tc": round(nnz / max(T, 1), 3), "sum_u": ab["sum_u"],
                 "unit_blocks": fmt.unit_blocks, "num_units": fmt.num_units,
-                "split_windows": fmt.num_split_windows,
+                "split_windows": fmt.num_split_windows, "guided": fmt.get_option("guided"),
+                "f4_plan": "selector" if args.selector else "rule",
+                "selector_predicted_ms": round(fmt.get_option("plan_makespan_ns") / 1e6, 4) or None,
                 "format_build_ms": round(build_ms_runs[-1], 3),
                 "format_build_first_call_ms": round(build_ms_runs[0], 3),
                 "format_build_x_spmm": round(build_ms_runs[-1] / kern_ms, 2)})
@@ -445,7 +450,7 @@ def headline_extras(args, cfg, N, dev, stream, flush, leg, x):
     M, K, nnz = cfg.M, cfg.K, len(x["ci"])
     sm = torch.cuda.get_device_properties(dev).multi_processor_count
     try:
-        leg["selector"] = dtc.selector_report(x["exp"]["row_window_offset"], sm)
+        leg["selector"] = dtc.selector_report(x["exp"]["row_window_offset"], sm, cfg.dtype, N)
     except Exception as e:  # noqa: BLE001
         leg["selector"] = {"error": str(e)}
     if args.tca == 1 or (args.tca < 0 and nnz < 10_000_000):

@@ -81,7 +81,7 @@ typedef struct {
     const int32_t* units;
 } dtc_format_view_t;
 
-/* Build options (zero-initialised = defaults; window_order documented at the field).
+/* Build options (zero-initialised = defaults; window_order, n_hint, selector documented at the fields).
  *   unit_blocks  target TC blocks per work unit (F4); 0 = auto from T, W and the SM count
  *   dedup_path   F1 per-window dedup: 0 auto, 1 force smem sort, 2 force chunked bitmap
  *                (both produce bit-identical formats; exposed for tests)
@@ -99,6 +99,12 @@ typedef struct {
      * ORIGINAL row order (e.g. the TCA order from dtc_tca_reorder).  NULL = identity.
      * Not a permutation -> DTC_ERR_INVALID. */
     const int32_t* row_perm;
+    /* B200 Selector (NEXT-4, dtc_selector_plan): with unit_blocks = 0 and selector = 1, F4 takes the
+     * unit size and guided tail whose simulated launch for N = n_hint columns (0 = 128) is shortest;
+     * selector = 0 keeps the fixed rule (U = clamp(2T/W, 64, 256), at most T/(24 SMs); guided as above).
+     * Same C either way (within tolerance; integer inputs bit-exact). */
+    int32_t n_hint;
+    int32_t selector;
 } dtc_build_opts_t;
 
 /* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on
@@ -177,7 +183,9 @@ typedef enum {
     DTC_OPT_HOST_ZERO_COPY = 5,
     DTC_OPT_SLICE_BYTES = 6,
     DTC_OPT_LAST_KERNEL = 100,
-    DTC_OPT_LAST_HOST_MODE = 101
+    DTC_OPT_LAST_HOST_MODE = 101,
+    DTC_OPT_GUIDED = 102,            /* read-only: 1 if F4 cut a guided tail */
+    DTC_OPT_PLAN_MAKESPAN_NS = 103   /* read-only: the Selector's simulated makespan (ns), 0 = fixed rule */
 } dtc_option_t;
 int dtc_format_set_option(dtc_handle_t h, int32_t option, int64_t value);
 int dtc_format_get_option(dtc_handle_t h, int32_t option, int64_t* value);
@@ -233,6 +241,49 @@ int dtc_graphconv_launches_per_call(void);
  * Errors: INVALID (odd or < 2 num_sms, occupancy outside 1..1024, non-monotone rwo). */
 int dtc_selector_ar(const int32_t* rwo_host, int64_t num_windows, int32_t num_sms, int32_t occupancy,
                     double* makespan_base, double* makespan_balanced, double* ar);
+
+/* ------------------------------------------------------------ B200 Selector (NEXT-4)
+ * The paper's Selector (§4.5.2) simulates its base kernel's thread-block
+ * schedule to decide whether balancing pays.  libdtc always runs TC-block-balanced F4 units, so
+ * the retargeted Selector decides how to cut them: it simulates, for each candidate unit size U
+ * (and with/without the guided tail), the launch of exactly the units F4 would emit -- dispatched
+ * in order onto num_sms x occupancy resident-CTA slots, each unit holding its slot for
+ * cta_ns + block_ns * nb (+ fixup_ns * (G + ceil(np/G)) on the last piece of a window split into
+ * np pieces, G = ceil(sqrt(np)) or np if np <= 4) -- and keeps the shortest makespan (ties: larger U).
+ * dtc_format_build_ex runs it when opts->selector = 1 and opts->unit_blocks = 0. */
+typedef struct {
+    int32_t num_sms;      /* SMs (148 on B200) */
+    int32_t occupancy;    /* resident CTAs per SM of the kernel that will run (measured) */
+    double cta_ns;        /* slot time of a CTA beyond its blocks (startup + epilogue) */
+    double block_ns;      /* slot time per TC block */
+    double fixup_ns;      /* per dependent partial load of a split-window fixup */
+} dtc_sched_model_t;
+typedef struct {
+    int32_t unit_blocks;  /* U */
+    int32_t guided;       /* 1 = guided tail (units of U/2 over the last ~4U blocks per SM) */
+    int64_t num_units;    /* units (CTAs per column group) of the plan; -1 = not evaluated */
+    double makespan_ns;   /* simulated makespan; -1 = not evaluated */
+} dtc_plan_t;
+
+/* Default B200 model for dtype and N on the CURRENT device: occupancy measured with
+ * cudaOccupancyMaxActiveBlocksPerMultiprocessor on the kernel dtc_spmm would launch for N,
+ * cta_ns 2500, block_ns = occupancy x 8 x (CTA columns) x elt / (62.8 B/ns per SM, the measured
+ * gather4 rate), fixup_ns 1000.  Errors: INVALID, CUDA (no device). */
+int dtc_sched_model(int32_t dtype, int64_t N, dtc_sched_model_t* m);
+
+/* HOST, pure: plan F4 for RowWindowOffset rwo_host[W+1].  cand_u[ncand] candidate unit sizes (>= 8;
+ * NULL / 0 = {16,24,32,48,64,96,128,192,256,384,512}); guided: 0 = try both, 1 = only with, -1 =
+ * only without the guided tail.  plans (may be NULL) receives 2*ncand entries, plan k = candidate
+ * k/2 with guided = k&1 (excluded plans have makespan -1); best receives the winner.
+ * Errors: INVALID (bad model, non-monotone rwo, candidate < 8). */
+int dtc_selector_plan(const int32_t* rwo_host, int64_t num_windows, const dtc_sched_model_t* m,
+                      const int32_t* cand_u, int32_t ncand, int32_t guided, dtc_plan_t* plans,
+                      dtc_plan_t* best);
+
+/* HOST, pure: simulated makespan (ns) of an explicit unit list (units_host int32[8*nu] in the
+ * dtc_format_export layout, dispatched in the given order) under model m.  Errors: INVALID. */
+int dtc_selector_simulate(const int32_t* units_host, int64_t nu, const dtc_sched_model_t* m,
+                          double* makespan_ns);
 
 /* ------------------------------------------------------------ distributed
  * One process per GPU (north_star).  Row windows are partitioned across ranks

@@ -41,7 +41,23 @@ class _View(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("window_order", _i32),
-                ("row_perm", _vp)]
+                ("row_perm", _vp), ("n_hint", _i32), ("selector", _i32)]
+
+
+class SchedModel(ctypes.Structure):
+    """dtc_sched_model_t: the B200 Selector's launch model."""
+    _fields_ = [("num_sms", _i32), ("occupancy", _i32), ("cta_ns", ctypes.c_double), ("block_ns", ctypes.c_double),
+                ("fixup_ns", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class _Plan(ctypes.Structure):
+    _fields_ = [("unit_blocks", _i32), ("guided", _i32), ("num_units", _i64), ("makespan_ns", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 class DtcError(RuntimeError):
@@ -84,6 +100,9 @@ def lib():
             L.dtc_graphconv.argtypes = [_vp, _vp, _i64, _vp, _i64, _vp, _i32, _vp, _vp, _vp]
             L.dtc_graphconv_launches_per_call.argtypes = []
             L.dtc_selector_ar.argtypes = [_vp, _i64, _i32, _i32, _vp, _vp, _vp]
+            L.dtc_sched_model.argtypes = [_i32, _i64, P(SchedModel)]
+            L.dtc_selector_plan.argtypes = [_vp, _i64, P(SchedModel), _vp, _i32, _i32, _vp, P(_Plan)]
+            L.dtc_selector_simulate.argtypes = [_vp, _i64, P(SchedModel), P(ctypes.c_double)]
             L.dtc_tca_reorder.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp]
             L.dtc_nccl_unique_id.argtypes = [_vp]
             L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
@@ -130,7 +149,7 @@ def launches_per_call() -> int:
 
 # per-handle launch options (include/dtc.h dtc_option_t)
 OPTIONS = {"kernel": 1, "persistent": 2, "first_records": 3, "host_chunks": 4, "host_zero_copy": 5,
-           "slice_bytes": 6, "last_kernel": 100, "last_host_mode": 101}
+           "slice_bytes": 6, "last_kernel": 100, "last_host_mode": 101, "guided": 102, "plan_makespan_ns": 103}
 KERNELS = {"auto": 0, "ldg": 1, "pad": 4}
 
 
@@ -183,16 +202,18 @@ class Format:
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
               unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None,
-              window_order: bool = False) -> "Format":
+              window_order: bool = False, n_hint: int = 0, selector: int = 0) -> "Format":
         """row_perm: optional CUDA int32 tensor [M], new row -> original row (e.g. tca_reorder);
-        C is still produced in the original row order."""
+        C is still produced in the original row order.  selector=1 (with unit_blocks=0): F4 cut by
+        the B200 Selector's plan for N = n_hint columns (dtc_selector_plan)."""
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
         h = ctypes.c_void_p()
         if row_perm is not None:
             import torch
             if row_perm.dtype != torch.int32 or not row_perm.is_cuda or row_perm.numel() != M:
                 raise TypeError("row_perm must be a CUDA int32 tensor of length M")
-        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm))
+        opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm),
+                     int(n_hint), int(selector))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value, device=rowptr.device.index or 0)
@@ -385,6 +406,50 @@ def selector_ar(rwo, num_sms: int = 148, occupancy: int = 6) -> dict:
            "dtc_selector_ar")
     return {"makespan_base": float(out[0]), "makespan_balanced": float(out[1]), "ar": float(out[2]),
             "num_sms": num_sms, "occupancy": occupancy}
+
+
+def sched_model(dtype="tf32", N: int = 128) -> SchedModel:
+    """The default B200 launch model for dtype and N on the current device (dtc_sched_model)."""
+    m = SchedModel()
+    _check(lib().dtc_sched_model(_dtype_code(dtype), int(N), ctypes.byref(m)), "dtc_sched_model")
+    return m
+
+
+def make_model(num_sms: int, occupancy: int, cta_ns: float, block_ns: float, fixup_ns: float) -> SchedModel:
+    return SchedModel(int(num_sms), int(occupancy), float(cta_ns), float(block_ns), float(fixup_ns))
+
+
+def selector_plan(rwo, model: SchedModel, candidates=None, guided: int = 0) -> dict:
+    """B200 Selector (dtc_selector_plan): every candidate plan's simulated makespan and the best."""
+    rwo = np.ascontiguousarray(rwo, dtype=np.int32)
+    cand = None if candidates is None else np.ascontiguousarray(candidates, dtype=np.int32)
+    nc = 11 if cand is None else len(cand)
+    plans = (_Plan * (2 * nc))()
+    best = _Plan()
+    _check(lib().dtc_selector_plan(rwo.ctypes.data_as(_vp), len(rwo) - 1, ctypes.byref(model),
+                                   None if cand is None else cand.ctypes.data_as(_vp), 0 if cand is None else nc,
+                                   int(guided), ctypes.cast(plans, _vp), ctypes.byref(best)), "dtc_selector_plan")
+    return {"best": best.as_dict(), "plans": [p.as_dict() for p in plans]}
+
+
+def selector_simulate(units, model: SchedModel) -> float:
+    """Simulated makespan (ns) of an explicit unit list [nu, 8] (dtc_selector_simulate)."""
+    u = np.ascontiguousarray(units, dtype=np.int32).reshape(-1, 8)
+    out = ctypes.c_double()
+    _check(lib().dtc_selector_simulate(u.ctypes.data_as(_vp), len(u), ctypes.byref(model), ctypes.byref(out)),
+           "dtc_selector_simulate")
+    return float(out.value)
+
+
+def selector_report(rwo, num_sms: int = 148, dtype="tf32", N: int = 128, occupancy_paper: int = 6) -> dict:
+    """The paper's AR (Eq. (1) model) and the B200 Selector's plan for this RowWindowOffset."""
+    ar = selector_ar(rwo, num_sms, occupancy_paper)
+    m = sched_model(dtype, N)
+    plan = selector_plan(rwo, m)
+    return {"paper_ar": round(ar["ar"], 3), "paper_rule_balanced": ar["ar"] > 1.2, "model": m.as_dict(),
+            "plan": plan["best"],
+            "candidates": {f"U{p['unit_blocks']}{'g' if p['guided'] else ''}": round(p["makespan_ns"] / 1e3, 2)
+                           for p in plan["plans"] if p["makespan_ns"] >= 0}}
 
 
 def tca_reorder(M: int, K: int, rowptr, colidx, sm_num: int = 148) -> np.ndarray:

@@ -23,9 +23,11 @@
 #include <cstring>
 #include <chrono>
 #include <new>
+#include <vector>
 
 #include "dtc_device.cuh"
 #include "dtc_internal.h"
+#include "dtc_sched.h"
 
 namespace dtc {
 
@@ -351,58 +353,7 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
 }
 
 // ---------------------------------------------------------------- F4
-// Work units: consecutive windows whose first TC block falls in
-// the same chunk form one unit; a window with more blocks than its chunk size is
-// split into near-equal pieces (each its own unit, deterministic fixup).  Chunk
-// sizes are "guided": U blocks, then U/2, U/4, U/8 over the last ~one wave of
-// blocks, so the CTAs dispatched last are short and the tail of the grid is even.
-struct Guide {
-    int64_t x[5];     // segment starts (x[4] = T)
-    int64_t sz[4];    // chunk size per segment
-    int64_t off[4];   // chunk-id offset per segment
-    __host__ __device__ int seg(int64_t v) const {
-        int k = 0;
-        while (k < 3 && v >= x[k + 1]) ++k;
-        return k;
-    }
-    __host__ __device__ int64_t chunk(int64_t v) const {
-        const int k = seg(v);
-        return off[k] + (v - x[k]) / sz[k];
-    }
-    __host__ __device__ int64_t size_at(int64_t v) const { return sz[seg(v)]; }
-};
-
-static Guide make_guide(int64_t T, int U, int64_t tail_span) {
-    Guide g;
-    int64_t A = tail_span > T ? T : tail_span;
-    g.x[0] = 0;
-    g.x[1] = T - A;
-    g.x[2] = T - A / 2;
-    g.x[3] = T - A / 4;
-    g.x[4] = T;
-    // sizes U, then U/2 for the rest of the tail (smaller units lose more to per-unit
-    // startup than they win at the end of the grid -- measured)
-    for (int k = 0; k < 4; ++k) {
-        const int64_t sz = k == 0 ? U : U / 2;
-        g.sz[k] = sz < 8 ? 8 : sz;
-    }
-    g.off[0] = 0;
-    for (int k = 1; k < 4; ++k) g.off[k] = g.off[k - 1] + (g.x[k] - g.x[k - 1] + g.sz[k - 1] - 1) / g.sz[k - 1];
-    return g;
-}
-
-// Pieces of a split window (nb > U blocks): at least U blocks each, and at most ~sqrt(nb/2) of them.
-// A piece costs ~nb/np block times (~0.5 us each) and the last arriver's fixup chains np dependent
-// partial loads (~1 us each), so the window's critical path nb/np * 0.5 + np is smallest near
-// np = sqrt(nb/2) (c2's hub windows: ~1,600 blocks -> 29 pieces instead of 100 at U = 16).
-__host__ __device__ __forceinline__ int64_t split_pieces(int64_t nb, int64_t U) {
-    const int64_t byU = (nb + U - 1) / U;
-    int64_t r = (int64_t)sqrt((double)nb * 0.5);
-    if (r < 1) r = 1;
-    while (2 * r * r < nb) ++r;   // ceil(sqrt(nb/2))
-    while (r > 1 && 2 * (r - 1) * (r - 1) >= nb) --r;
-    return byU < r ? byU : r;
-}
+// F4 rules (Guide, split_pieces): dtc_sched.h, shared with the Selector's host simulation.
 
 __global__ void k_units_count(int64_t W, const int32_t* __restrict__ rwo, Guide gd,
                               int64_t* __restrict__ cnt, int64_t* __restrict__ split,
@@ -696,12 +647,28 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         st.mark("F3 fill");
         // F4: work units
         int U = (opts && opts->unit_blocks > 0) ? opts->unit_blocks : auto_unit_blocks(T, W);
-        h->unit_blocks = U;
         // guided tail (units of U/2 over about half a wave): opts->guided 1 = on, -1 = off, 0 = auto:
         // on when the launch is only a few waves long (< 8 waves of 6 CTAs per SM), where the last
         // partial wave is a large part of it (arxiv-shaped c2: +5% measured; c3-c5 have 20-300 waves)
         const int gopt = opts ? opts->guided : 0;
-        const bool guided = gopt > 0 || (gopt == 0 && T < (int64_t)8 * 6 * num_sms() * U);
+        bool guided = gopt > 0 || (gopt == 0 && T < (int64_t)8 * 6 * num_sms() * U);
+        // B200 Selector (NEXT-4, dtc_selector.cu): with no unit size given, simulate the launch of
+        // every candidate plan (U x guided tail) for the expected N and keep the shortest
+        const int sel = opts ? opts->selector : 0;
+        if (!(opts && opts->unit_blocks > 0) && sel > 0 && T > 0) {
+            std::vector<int32_t> hrwo((size_t)W + 1);
+            TRYC(cudaMemcpyAsync(hrwo.data(), h->rwo, (W + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            TRYC(cudaStreamSynchronize(s));
+            dtc_sched_model_t m;
+            TRY(sched_model(h->dtype, (opts && opts->n_hint > 0) ? opts->n_hint : 128, &m));
+            dtc_plan_t best;
+            TRY(selector_plan(hrwo.data(), W, m, nullptr, 0, gopt, nullptr, &best));
+            U = best.unit_blocks;
+            guided = best.guided != 0;
+            h->plan_makespan_ns = best.makespan_ns;
+        }
+        h->unit_blocks = U;
+        h->guided = guided ? 1 : 0;
         const int64_t tail = guided ? (int64_t)num_sms() * 4 * U : 0;
         const Guide gd = make_guide(T, U, tail);
         if (W > 0) {

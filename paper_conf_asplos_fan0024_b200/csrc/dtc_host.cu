@@ -212,6 +212,8 @@ extern "C" int dtc_format_get_option(dtc_handle_t h, int32_t option, int64_t* va
         case DTC_OPT_SLICE_BYTES: *value = h->opt.slice_bytes; return DTC_OK;
         case DTC_OPT_LAST_KERNEL: *value = h->last_kernel; return DTC_OK;
         case DTC_OPT_LAST_HOST_MODE: *value = h->last_host_mode; return DTC_OK;
+        case DTC_OPT_GUIDED: *value = h->guided; return DTC_OK;
+        case DTC_OPT_PLAN_MAKESPAN_NS: *value = (int64_t)(h->plan_makespan_ns + 0.5); return DTC_OK;
         default: set_error("option %d is unknown", (int)option); return DTC_ERR_INVALID;
     }
 }

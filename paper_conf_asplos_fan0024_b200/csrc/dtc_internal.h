@@ -39,6 +39,8 @@ struct dtc_format {
     int64_t M = 0, K = 0, nnz = 0, W = 0, T = 0;
     int32_t dtype = 0;
     int32_t unit_blocks = 0;
+    int32_t guided = 0;               // F4 guided tail in use
+    double plan_makespan_ns = 0.0;    // Selector's simulated makespan of the chosen plan (0 = rule)
     int device = 0;
     int32_t* rwo = nullptr;      // [W+1]
     int32_t* tco = nullptr;      // [T+1]
@@ -137,6 +139,19 @@ int num_sms();
 // SpMM kernel launcher (dtc_spmm.cu)
 int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, int64_t ldc,
                 cudaStream_t s);
+
+// padded-path geometry and measured occupancy for N columns (dtc_spmm.cu), used by the Selector
+struct PadGeometry {
+    int seg, slices;
+    int64_t cta_cols;
+};
+PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes);
+int pad_occupancy(int dtype, int64_t N);
+
+// B200 Selector (dtc_selector.cu): simulate the F4 units of each candidate plan, return the best
+int selector_plan(const int32_t* rwo, int64_t W, const dtc_sched_model_t& m, const int32_t* cand, int ncand,
+                  int guided_opt, dtc_plan_t* plans, dtc_plan_t* best);
+int sched_model(int dtype, int64_t N, dtc_sched_model_t* m);
 
 // internal build used by the distributed layer: optional row range of the csr
 int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s,

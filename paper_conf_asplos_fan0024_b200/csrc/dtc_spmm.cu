@@ -29,6 +29,7 @@
 #include <vector>
 
 #include "dtc_internal.h"
+#include "dtc_sched.h"
 
 namespace dtc {
 
@@ -112,6 +113,15 @@ __device__ __forceinline__ int frag_slot(int id) {
     }
 }
 
+// FP16 block pairing (reading C15): step i of a unit pairs TC blocks i and i+1 when both exist, belong
+// to one window, and do not straddle a kFp16PairSpan-block boundary of the unit (the padded kernel's
+// A batches and the register-gather kernel's A chunks are multiples of it) -- one rule for both
+// kernels, so they compute identical sums and C(:, j) does not depend on which kernel N selects.
+constexpr int kFp16PairSpan = 16;
+__device__ __forceinline__ bool fp16_pair(int dt, int i, int nblocks, int bb, int next_end) {
+    return dt == DTC_FP16 && i + 1 < nblocks && bb + i + 1 != next_end && (i + 1) % kFp16PairSpan != 0;
+}
+
 struct alignas(16) V16 {
     uint32_t w[4];
 };
@@ -188,12 +198,6 @@ __device__ __forceinline__ void store_tile(float* __restrict__ C, int64_t ldc, i
 // chain made the last arriver of a hub window the tail of the launch).  Counters live at
 // ctr0[slot * cstride] (one per slot and warp column slice): group g at its first slot, the window
 // at slot_base + 1 (never a group's first slot when there are >= 2 groups); all self-resetting.
-__device__ __forceinline__ int fixup_group(int np) {
-    if (np <= 4) return np;
-    int g = 1;
-    while (g * g < np) ++g;
-    return g;
-}
 
 template <int NJ, int QPC, int CSTRIDE>
 __device__ __forceinline__ void fixup_write(float (&acc)[NJ][4], float* __restrict__ ws, int64_t slot, int64_t npad,
@@ -509,60 +513,79 @@ k_spmm_ldg(const Unit* __restrict__ units, const int32_t* __restrict__ rwo, cons
                 }
             }
         }
-        for (int i0 = 0; i0 < nblocks; i0 += P) {
+        static_assert(P == 1, "the block-pair step below assumes a one-block register prefetch");
+        static_assert(S % kFp16PairSpan == 0, "FP16 pairs never straddle an A chunk");
+        for (int i = 0; i < nblocks;) {
+            const int c = i / S, j = i % S;
+            // FP16: blocks i, i+1 of one window feed one m16n8k16 (same pairing rule as k_spmm_pad,
+            // so both kernels compute identical sums); block i+1's B rows are gathered here (its
+            // fragment and ids are in the same A chunk), the next step's one block ahead as usual
+            const bool pair = fp16_pair(DT, i, nblocks, u.bb, next_end);
+            const int nx = i + (pair ? 2 : 1);
+            if (active) {
+                const uint32_t* fr = s_frag + (c & 1) * S * 32 * FW + j * 32 * FW;
+                if (DT == DTC_TF32) {
+                    const uint4 av = reinterpret_cast<const uint4*>(fr)[lane];
+                    const uint32_t a[4] = {av.x, av.y, av.z, av.w};
 #pragma unroll
-            for (int q = 0; q < P; ++q) {
-                const int i = i0 + q;
-                if (i < nblocks) {
-                    const int c = i / S, j = i % S;
-                    if (active) {
-                        const uint32_t* fr = s_frag + (c & 1) * S * 32 * FW + j * 32 * FW;
-                        if (DT == DTC_TF32) {
-                            const uint4 av = reinterpret_cast<const uint4*>(fr)[lane];
-                            const uint32_t a[4] = {av.x, av.y, av.z, av.w};
+                    for (int cw = 0; cw < CW; ++cw)
 #pragma unroll
-                            for (int cw = 0; cw < CW; ++cw)
+                        for (int jj = 0; jj < NJ1; ++jj)
+                            mma_tf32(acc[cw * NJ1 + jj], a, b0[0][cw].w[jj], b1[0][cw].w[jj]);
+                } else if (pair) {
+                    const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
+                    const uint2 av2 = reinterpret_cast<const uint2*>(fr + 32 * FW)[lane];
+                    const uint32_t a[4] = {av.x, av.y, av2.x, av2.y};
+                    const int2 id2 = ids_of(i + 1);
 #pragma unroll
-                                for (int jj = 0; jj < NJ1; ++jj)
-                                    mma_tf32(acc[cw * NJ1 + jj], a, b0[q][cw].w[jj], b1[q][cw].w[jj]);
-                        } else {
-                            const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
-                            const uint32_t a[2] = {av.x, av.y};
+                    for (int cw = 0; cw < CW; ++cw) {
+                        const V16 z0 = gather(id2.x, cw), z1 = gather(id2.y, cw);
 #pragma unroll
-                            for (int cw = 0; cw < CW; ++cw)
-#pragma unroll
-                                for (int jj = 0; jj < NJ1; ++jj) {
-                                    const uint32_t bb = __byte_perm(b0[q][cw].w[jj >> 1], b1[q][cw].w[jj >> 1],
-                                                                    (jj & 1) ? 0x7632 : 0x5410);
-                                    mma_f16(acc[cw * NJ1 + jj], a, bb);
-                                }
+                        for (int jj = 0; jj < NJ1; ++jj) {
+                            const uint32_t sel = (jj & 1) ? 0x7632 : 0x5410;
+                            const uint32_t bb0 = __byte_perm(b0[0][cw].w[jj >> 1], b1[0][cw].w[jj >> 1], sel);
+                            const uint32_t bb1 = __byte_perm(z0.w[jj >> 1], z1.w[jj >> 1], sel);
+                            mma_f16_k16(acc[cw * NJ1 + jj], a, bb0, bb1);
                         }
-                        if (i + P < nblocks) {
-                            const int2 id = ids_of(i + P);
+                    }
+                } else {
+                    const uint2 av = reinterpret_cast<const uint2*>(fr)[lane];
+                    const uint32_t a[2] = {av.x, av.y};
 #pragma unroll
-                            for (int cw = 0; cw < CW; ++cw) {
-                                b0[q][cw] = gather(id.x, cw);
-                                b1[q][cw] = gather(id.y, cw);
-                            }
-                        }
-                        if (u.bb + i + 1 == next_end) {
-                            store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+                    for (int cw = 0; cw < CW; ++cw)
 #pragma unroll
-                            for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
-                            ++cur;
-                            while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
-                                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
-                                ++cur;
-                            }
-                            next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+                        for (int jj = 0; jj < NJ1; ++jj) {
+                            const uint32_t bb = __byte_perm(b0[0][cw].w[jj >> 1], b1[0][cw].w[jj >> 1],
+                                                            (jj & 1) ? 0x7632 : 0x5410);
+                            mma_f16(acc[cw * NJ1 + jj], a, bb);
                         }
+                }
+                if (nx < nblocks) {
+                    const int2 id = ids_of(nx);
+#pragma unroll
+                    for (int cw = 0; cw < CW; ++cw) {
+                        b0[0][cw] = gather(id.x, cw);
+                        b1[0][cw] = gather(id.y, cw);
                     }
                 }
             }
-            const int nxt = i0 + P;   // S is a multiple of P: chunk boundaries fall between groups
-            if (nxt % S == 0 && nxt < nblocks) {
+            // every warp (active or not) tracks the window ends, so the step -- and with it the
+            // chunk-boundary barriers below -- stays CTA-uniform
+            if (u.bb + nx == next_end) {
+                if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+#pragma unroll
+                for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+                ++cur;
+                while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
+                    if (active) store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                    ++cur;
+                }
+                next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
+            }
+            // a step never straddles a chunk (pairs stay inside a kFp16PairSpan-aligned span, which divides S)
+            i = nx;
+            if (i % S == 0 && i < nblocks) {
                 // chunk boundary (CTA-uniform): finish chunk c+1's fragments, recycle buffer c&1
-                const int c = nxt / S - 1;
                 ent_store_n((c + 1) & 1, chunk_nb(c + 1));
                 __syncthreads();
                 if (c + 2 < nchunks) meta_store(c + 2, c & 1);
@@ -621,6 +644,7 @@ constexpr int pad_stages() {
 // the) batch's TCValues -- contiguous, TCOffset[b0] .. TCOffset[b0+16] -- and one of its 16
 // occupancy masks, double buffered.
 constexpr int kPadBatch = 16;
+static_assert(kPadBatch % kFp16PairSpan == 0, "FP16 pairs never straddle an A batch");
 // per-unit side record for the first batch (DTC_OPT_FIRST_RECORDS): kPadBatch x 8 SparseAtoB ids
 // (-1 past the unit), TCOffset[bb], TCOffset[bb + min(kPadBatch, nb)], end of the first window, pad
 constexpr int kFirstRec = kPadBatch * 8 + 4;
@@ -980,7 +1004,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             const int gi = gi0 + i, s = gi % R;
             // FP16: two TC blocks of one window feed one m16n8k16 (k = block i's 8 columns, then
             // block i+1's -- the k16 A/B fragments are exactly the two k8 fragments side by side)
-            const bool pair = DT == DTC_FP16 && i + 1 < nblocks && u.bb + i + 1 != next_end;
+            const bool pair = fp16_pair(DT, i, nblocks, u.bb, next_end);
             uint32_t a[FW], a2[FW];
             afrag(i, gc0, a);
             if (pair) afrag(i + 1, gc0, a2);
@@ -1267,6 +1291,43 @@ static cudaError_t dispatch_pad(int slices, const LaunchArgs& a, const CUtensorM
     return slices >= 2 ? launch_pad<DT, 2, 4, VEC>(a, map) : launch_pad<DT, 1, 4, VEC>(a, map);
 }
 
+// Padded-path geometry for N columns: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB,
+// else 512 B; <= 2 slices (seg/2 consumer warps each) per CTA.
+PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes) {
+    const int elt = elt_size(dtype);
+    PadGeometry g;
+    g.seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : 4;
+    if (slice_bytes == 512) g.seg = 4;
+    if (slice_bytes == 1024 && (N * elt) % 8 == 0) g.seg = 8;
+    const int64_t slice_cols = g.seg * 128 / elt;
+    const int64_t nsl = (N + slice_cols - 1) / slice_cols;
+    g.slices = nsl >= 2 ? 2 : 1;
+    g.cta_cols = g.slices * slice_cols;
+    return g;
+}
+
+// Resident CTAs per SM of the padded kernel dtc_spmm would launch for N columns (vector C path), on
+// the current device -- the measured occupancy the Selector plans with.
+int pad_occupancy(int dtype, int64_t N) {
+    const PadGeometry g = pad_geometry(dtype, N, 0);
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return -1; }
+    auto occ = [&](auto kern, int sl, int seg) -> int {
+        static KernelState ks[8];
+        const int idx = (dtype == DTC_FP16 ? 4 : 0) + (sl - 1) * 2 + (seg == 8 ? 1 : 0);
+        const int threads = (sl * seg / 2 + 1) * 32;
+        const size_t smem = sl == 1 ? (seg == 4 ? pad_smem_bytes<1, 4>() : pad_smem_bytes<1, 8>())
+                                    : (seg == 4 ? pad_smem_bytes<2, 4>() : pad_smem_bytes<2, 8>());
+        return kernel_setup(kern, threads, smem, ks[idx], dev);
+    };
+    if (dtype == DTC_FP16) {
+        if (g.seg == 8) return g.slices >= 2 ? occ(k_spmm_pad<DTC_FP16, 2, 8, true>, 2, 8) : occ(k_spmm_pad<DTC_FP16, 1, 8, true>, 1, 8);
+        return g.slices >= 2 ? occ(k_spmm_pad<DTC_FP16, 2, 4, true>, 2, 4) : occ(k_spmm_pad<DTC_FP16, 1, 4, true>, 1, 4);
+    }
+    if (g.seg == 8) return g.slices >= 2 ? occ(k_spmm_pad<DTC_TF32, 2, 8, true>, 2, 8) : occ(k_spmm_pad<DTC_TF32, 1, 8, true>, 1, 8);
+    return g.slices >= 2 ? occ(k_spmm_pad<DTC_TF32, 2, 4, true>, 2, 4) : occ(k_spmm_pad<DTC_TF32, 1, 4, true>, 1, 4);
+}
+
 // RAII: make the handle's device current for the duration of a call
 struct DeviceGuard {
     int prev = -1;
@@ -1299,21 +1360,16 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     memset(&map, 0, sizeof(map));
     const bool tma_ok = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && ((N * elt) % 4 == 0) &&
                         h->K < (int64_t(1) << 31) && N < (int64_t(1) << 31);
-    // padded path: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB, else 512 B
-    int seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : 4;
-    if (h->opt.slice_bytes == 512) seg = 4;
-    if (h->opt.slice_bytes == 1024 && (N * elt) % 8 == 0) seg = 8;
+    const PadGeometry pg = pad_geometry(h->dtype, N, h->opt.slice_bytes);
+    const int seg = pg.seg;
     const int te = ((N * elt) % 8 == 0) ? 8 : 4;
     bool pad = h->opt.kernel != 1 && tma_ok && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg, te);
     int64_t cta_cols, slices = 1;
     int warps = 1;
     const int colw_ldg = (h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW) * kLdgColChunks;
     if (pad) {
-        // slices (of seg x 128 bytes of a B row) per CTA: seg/2 consumer warps each, <= 2 slices
-        const int64_t slice_cols = seg * 128 / elt;
-        const int64_t nsl = (N + slice_cols - 1) / slice_cols;
-        slices = nsl >= 2 ? 2 : 1;
-        cta_cols = slices * slice_cols;
+        slices = pg.slices;
+        cta_cols = pg.cta_cols;
     } else {
         const int64_t need = (N + colw_ldg - 1) / colw_ldg;
         warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
