@@ -105,6 +105,11 @@ typedef struct {
      * Same C either way (within tolerance; integer inputs bit-exact). */
     int32_t n_hint;
     int32_t selector;
+    /* transpose = 1: condense A^T (K x M) instead of A -- the rows of A^T are A's columns, in the
+     * canonical order (A's CSR is validated first; then a GPU radix sort by (column, row) gives A^T's
+     * CSR) -- e.g. the handle for the GCN backward dH = A^T dAH (NEXT-3).  Not combinable with
+     * row_perm (INVALID). */
+    int32_t transpose;
 } dtc_build_opts_t;
 
 /* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on

@@ -41,7 +41,7 @@ class _View(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("window_order", _i32),
-                ("row_perm", _vp), ("n_hint", _i32), ("selector", _i32)]
+                ("row_perm", _vp), ("n_hint", _i32), ("selector", _i32), ("transpose", _i32)]
 
 
 class SchedModel(ctypes.Structure):
@@ -202,10 +202,12 @@ class Format:
     @classmethod
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
               unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None,
-              window_order: bool = False, n_hint: int = 0, selector: int = 0) -> "Format":
+              window_order: bool = False, n_hint: int = 0, selector: int = 0,
+              transpose: bool = False) -> "Format":
         """row_perm: optional CUDA int32 tensor [M], new row -> original row (e.g. tca_reorder);
         C is still produced in the original row order.  selector=1 (with unit_blocks=0): F4 cut by
-        the B200 Selector's plan for N = n_hint columns (dtc_selector_plan)."""
+        the B200 Selector's plan for N = n_hint columns (dtc_selector_plan).  transpose=True condenses
+        A^T (K x M) from A's CSR (e.g. for the GCN backward)."""
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
         h = ctypes.c_void_p()
         if row_perm is not None:
@@ -213,7 +215,7 @@ class Format:
             if row_perm.dtype != torch.int32 or not row_perm.is_cuda or row_perm.numel() != M:
                 raise TypeError("row_perm must be a CUDA int32 tensor of length M")
         opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm),
-                     int(n_hint), int(selector))
+                     int(n_hint), int(selector), int(bool(transpose)))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value, device=rowptr.device.index or 0)

@@ -25,6 +25,8 @@
 #include <new>
 #include <vector>
 
+#include <cub/device/device_radix_sort.cuh>
+
 #include "dtc_device.cuh"
 #include "dtc_internal.h"
 #include "dtc_sched.h"
@@ -261,6 +263,41 @@ __global__ void k_perm_copy(int64_t M, const int32_t* __restrict__ perm, const i
     }
 }
 
+// ---------------------------------------------------------------- optional transpose
+// (dtc_build_opts_t.transpose): the ME-TCF of A^T -- e.g. for the GCN backward dH = A^T dAH -- from
+// A's CSR on the GPU: one 64-bit key (column << rbits | row) per non-zero, a radix sort (CUB, a
+// plain library sort of the one-time build) keyed by (column, row) gives A^T's canonical CSR
+// (rows = A's columns, entries by ascending original row), values gathered by the sorted index.
+__global__ void k_tr_keys(int64_t M, int64_t nnz, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ ci,
+                          int rbits, uint64_t* __restrict__ keys, int32_t* __restrict__ idx) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = warp; r < M; r += nwarps) {
+        const int64_t lo = clamp64(rowptr[r], 0, nnz), hi = clamp64(rowptr[r + 1], 0, nnz);
+        for (int64_t p = lo + lane; p < hi; p += 32) {
+            keys[p] = ((uint64_t)(uint32_t)ci[p] << rbits) | (uint64_t)r;
+            idx[p] = (int32_t)p;
+        }
+    }
+}
+template <class V>
+__global__ void k_tr_fill(int64_t nnz, int64_t Mt, int rbits, const uint64_t* __restrict__ keys,
+                          const int32_t* __restrict__ idx, const V* __restrict__ vin, int32_t* __restrict__ rowptr_t,
+                          int32_t* __restrict__ ci_t, V* __restrict__ v_t) {
+    const uint64_t rmask = (uint64_t(1) << rbits) - 1;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e <= nnz; e += (int64_t)gridDim.x * blockDim.x) {
+        // row c of A^T starts at the first sorted key of column c: fill rowptr_t[prev+1 .. c]
+        const int64_t c = e < nnz ? (int64_t)(keys[e] >> rbits) : Mt;
+        const int64_t prev = e > 0 ? (int64_t)(keys[e - 1] >> rbits) : -1;
+        for (int64_t k = prev + 1; k <= c; ++k) rowptr_t[k] = (int32_t)e;
+        if (e < nnz) {
+            ci_t[e] = (int32_t)(keys[e] & rmask);
+            v_t[e] = vin[idx[e]];
+        }
+    }
+}
+
 // ---------------------------------------------------------------- F2/F3
 __global__ void k_to_i32(const int64_t* __restrict__ in, int32_t* __restrict__ out, int64_t n) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -466,7 +503,13 @@ struct BuildTemps {
     int32_t* prow32 = nullptr;   // row_perm: permuted rowptr
     int32_t* pcol = nullptr;     // row_perm: permuted colidx
     uint8_t* pval = nullptr;     // row_perm: permuted values
+    uint64_t* tkeys = nullptr;   // transpose: sort keys (in / out)
+    uint64_t* tkeys2 = nullptr;
+    int32_t* tidx = nullptr;     // transpose: nnz index (in / out)
+    int32_t* tidx2 = nullptr;
+    uint8_t* tsort = nullptr;    // transpose: CUB temp storage
     void release(cudaStream_t s) {
+        dfree(tkeys, s); dfree(tkeys2, s); dfree(tidx, s); dfree(tidx2, s); dfree(tsort, s);
         dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s);
         dfree(scan_tmp, s); dfree(cnt, s); dfree(ucnt, s); dfree(usplit, s);
         dfree(uslots, s);
@@ -528,11 +571,15 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         return DTC_ERR_CUDA;
     }
     const int mode = opts ? opts->dedup_path : 0;
-    const int64_t W = (M + kWindow - 1) / kWindow;
+    const bool transpose = opts && opts->transpose;
+    if (transpose && opts->row_perm) { set_error("transpose and row_perm cannot be combined"); return DTC_ERR_INVALID; }
+    // the condensed matrix: A (M x K) or A^T (K x M)
+    const int64_t Mc = transpose ? K : M, Kc = transpose ? M : K;
+    const int64_t W = (Mc + kWindow - 1) / kWindow;
 
     dtc_format* h = new (std::nothrow) dtc_format();
     if (!h) { set_error("host OOM"); return DTC_ERR_OOM; }
-    h->M = M; h->K = K; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
+    h->M = Mc; h->K = Kc; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
     cudaGetDevice(&h->device);
     BuildTemps t;
     dtc_csr_t pcsr;   // permuted CSR view (row_perm)
@@ -581,17 +628,70 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             pcsr.vals = t.pval;
             csr = &pcsr;
         }
+        if (transpose && nnz > 0) {
+            // validate A itself (its keys must be in range), then build A^T's CSR and condense that
+            k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, t.flags);
+            TRYC(cudaMemcpyAsync(&t.host[1], t.flags, sizeof(int), cudaMemcpyDeviceToHost, s));
+            TRYC(cudaStreamSynchronize(s));
+            const int f0 = (int)(t.host[1] & 0xffffffff);
+            if (f0) {
+                if (f0 & F_INVALID) { set_error("malformed rowptr"); rc = DTC_ERR_INVALID; }
+                else if (f0 & F_RANGE) { set_error("column index out of [0, K)"); rc = DTC_ERR_RANGE; }
+                else if (f0 & F_DUPLICATE) { set_error("duplicate column within a row"); rc = DTC_ERR_DUPLICATE; }
+                else { set_error("columns not ascending within a row"); rc = DTC_ERR_UNSORTED; }
+                goto fail;
+            }
+            int rbits = 1;
+            while ((int64_t(1) << rbits) < M) ++rbits;
+            int cbits = 1;
+            while ((int64_t(1) << cbits) < K) ++cbits;
+            TRY(dalloc(&t.tkeys, nnz, s));
+            TRY(dalloc(&t.tkeys2, nnz, s));
+            TRY(dalloc(&t.tidx, nnz, s));
+            TRY(dalloc(&t.tidx2, nnz, s));
+            k_tr_keys<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, nnz, csr->rowptr, csr->colidx, rbits, t.tkeys, t.tidx);
+            size_t tb = 0;
+            TRYC(cub::DeviceRadixSort::SortPairs(nullptr, tb, t.tkeys, t.tkeys2, t.tidx, t.tidx2, (int)nnz, 0,
+                                                 rbits + cbits, s));
+            TRY(dalloc(&t.tsort, tb, s));
+            TRYC(cub::DeviceRadixSort::SortPairs(t.tsort, tb, t.tkeys, t.tkeys2, t.tidx, t.tidx2, (int)nnz, 0,
+                                                 rbits + cbits, s));
+            TRY(dalloc(&t.prow32, Mc + 1, s));
+            TRY(dalloc(&t.pcol, nnz, s));
+            TRY(dalloc(&t.pval, (size_t)nnz * elt_size(h->dtype), s));
+            if (h->dtype == DTC_FP16)
+                k_tr_fill<uint16_t><<<grid_for(nnz + 1, 256, 148 * 64), 256, 0, s>>>(
+                    nnz, Mc, rbits, t.tkeys2, t.tidx2, (const uint16_t*)csr->vals, t.prow32, t.pcol, (uint16_t*)t.pval);
+            else
+                k_tr_fill<uint32_t><<<grid_for(nnz + 1, 256, 148 * 64), 256, 0, s>>>(
+                    nnz, Mc, rbits, t.tkeys2, t.tidx2, (const uint32_t*)csr->vals, t.prow32, t.pcol, (uint32_t*)t.pval);
+            TRYC(cudaGetLastError());
+            dfree(t.tkeys, s); dfree(t.tkeys2, s); dfree(t.tidx, s); dfree(t.tidx2, s); dfree(t.tsort, s);
+            pcsr = *csr;
+            pcsr.M = Mc; pcsr.K = Kc;
+            pcsr.rowptr = t.prow32;
+            pcsr.colidx = t.pcol;
+            pcsr.vals = t.pval;
+            csr = &pcsr;
+        } else if (transpose) {
+            TRY(dalloc(&t.prow32, Mc + 1, s));
+            TRYC(cudaMemsetAsync(t.prow32, 0, (Mc + 1) * sizeof(int32_t), s));
+            pcsr = *csr;
+            pcsr.M = Mc; pcsr.K = Kc;
+            pcsr.rowptr = t.prow32;
+            csr = &pcsr;
+        }
         st.mark("setup+temp alloc");
         // F0
-        if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, t.flags);
+        if (Mc > 0) k_validate<<<grid_for(Mc * 32, 256, 148 * 64), 256, 0, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, t.flags);
         st.mark("F0 validate");
         // F1
         if (W > 0) {
-            k_dedup_sort<<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, mode,
+            k_dedup_sort<<<(unsigned)W, kSortThreads, 0, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
                                                              t.u, t.nb, t.uniq, t.rank);
             const size_t bm_smem = 2 * kBmWords * sizeof(uint32_t);
             TRYC(cudaFuncSetAttribute(k_dedup_bitmap, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
-            k_dedup_bitmap<<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, mode,
+            k_dedup_bitmap<<<(unsigned)W, kBmThreads, bm_smem, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
                                                                    t.u, t.nb, t.uniq, t.rank);
         }
         TRYC(cudaGetLastError());
@@ -634,11 +734,11 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             TRYC(cudaMemsetAsync(h->mask, 0, 4 * T * sizeof(uint32_t), s));
             if (h->dtype == DTC_FP16)
                 k_fill_window<uint16_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint16_t*)csr->vals,
+                    W, Mc, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint16_t*)csr->vals,
                     h->tco, h->lid, (uint16_t*)h->vals, h->atob);
             else
                 k_fill_window<uint32_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, M, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint32_t*)csr->vals,
+                    W, Mc, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint32_t*)csr->vals,
                     h->tco, h->lid, (uint32_t*)h->vals, h->atob);
         } else {
             TRYC(cudaMemsetAsync(h->tco, 0, sizeof(int32_t), s));
