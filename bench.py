@@ -456,14 +456,14 @@ def headline_extras(args, cfg, N, dev, stream, flush, leg, x):
     if args.tca == 1 or (args.tca < 0 and nnz < 10_000_000):
         try:
             t0 = time.perf_counter()
-            perm = dtc.tca_reorder(M, K, x["rp"], x["ci"], sm)
+            perm, tinfo = dtc.tca_reorder_checked(M, K, x["rp"], x["ci"], sm)
             reorder_s = time.perf_counter() - t0
             perm_d = torch.from_numpy(perm).to(dev)
             fmt_t = dtc.Format.build(x["rp_d"], x["ci_d"], x["v_d"], M, K, dtype=cfg.dtype, row_perm=perm_d)
             C_t = torch.empty((M, N), dtype=torch.float32, device=dev)
             ms_t = time_loop(lambda: fmt_t.spmm(B_d, C_t), max(10, min(args.steps, 50)), 3, stream, flush)
             tms = statistics.mean(ms_t)
-            leg["tca"] = {"value": round(x["flops"] / (tms * 1e-3) / 1e9, 2), "unit": UNIT,
+            leg["tca"] = {"value": round(x["flops"] / (tms * 1e-3) / 1e9, 2), "unit": UNIT, **tinfo,
                           "ms_per_step": round(tms, 5), "num_tc_blocks": fmt_t.num_tc_blocks,
                           "reorder_host_s": round(reorder_s, 3), "speedup_vs_unordered": round(x["kern_ms"] / tms, 3),
                           "matches_unordered": bool(torch.allclose(C_t, C_d, rtol=1e-2, atol=1e-2))}

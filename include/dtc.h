@@ -216,6 +216,14 @@ void dtc_format_destroy(dtc_handle_t h);   /* NULL-safe; frees all device memory
 int dtc_tca_reorder(int64_t M, int64_t K, const int32_t* rowptr_host, const int32_t* colidx_host,
                     int32_t sm_num, int32_t* perm_host);
 
+/* dtc_tca_reorder, then keep it only if it pays: NumTCBlock of the reordered and of
+ * the original row order are counted on the host; when the reordering does not lower it (e.g. a
+ * banded matrix already in its best order) perm is set to the identity.  T_identity, T_reordered
+ * (the counts) and applied (1 if perm is the TCA order) may each be NULL.  Errors: as above. */
+int dtc_tca_reorder_checked(int64_t M, int64_t K, const int32_t* rowptr_host, const int32_t* colidx_host,
+                            int32_t sm_num, int32_t* perm_host, int64_t* T_identity, int64_t* T_reordered,
+                            int32_t* applied);
+
 /* ------------------------------------------------------------ GraphConv (NEXT-3)
  * One GCN layer, §5.4 Eq. (2): Y = act((A x H) x W + b), in the
  * paper's order: AH = A*H by dtc_spmm (this library's kernel), then the dense
@@ -231,6 +239,28 @@ int dtc_graphconv(dtc_handle_t h, const void* H, int64_t F_in, const float* W, i
                   const float* bias, int32_t act, float* AH, float* Y, void* stream);
 /* Kernels one dtc_graphconv launches at least (SpMM + GEMM; cuBLASLt may add a reduction). */
 int dtc_graphconv_launches_per_call(void);
+
+/* Backward of one GraphConv layer Y = act(Z), Z = (A x H) x W + b (chain rule on Eq. (2)):
+ *   dZ  = dY * act'(Z)   (ReLU: 1 where Y > 0, else 0 -- the mask is read from Y; identity: dY)
+ *   dW  = AH^T dZ        (F_in x F_out)      cuBLASLt TF32, FP32 accumulate
+ *   db  = sum_rows dZ    (F_out; may be NULL) deterministic fixed-order reduction
+ *   dAH = dZ W^T         (M x F_in)          cuBLASLt TF32
+ *   dH  = A^T dAH        (K x F_in; may be NULL to skip) -- DTC-SpMM on ht, the ME-TCF of A^T built
+ *                        by dtc_format_build_ex with opts.transpose = 1 (TF32 handles only)
+ * AH, Y are the forward's; dZ (M x F_out) is caller workspace and may alias dY.  All device fp32
+ * row-major.  Errors: INVALID (shapes/handles), UNSUPPORTED (FP16 A^T), OOM, CUDA. */
+int dtc_graphconv_backward(dtc_handle_t h, dtc_handle_t ht, const float* AH, const float* W, int64_t F_in,
+                           int64_t F_out, int32_t act, const float* Y, const float* dY, float* dZ, float* dW,
+                           float* db, float* dAH, float* dH, void* stream);
+
+/* Training-step helpers for a GCN on top of the layer (NEXT-3):
+ * dtc_softmax_xent: loss (device scalar) = mean_i [log sum_c exp(z_ic) - z_i,label_i] over M rows of
+ * logits (M x num_classes, fp32), dlogits = (softmax(z_i) - onehot(label_i)) / M; labels int32[M] in
+ * [0, num_classes) (INVALID otherwise).  Synchronises `stream` (to report bad labels).
+ * dtc_sgd_update: param[i] -= lr * grad[i], i < n.  Errors: INVALID, OOM, CUDA. */
+int dtc_softmax_xent(const float* logits, const int32_t* labels, int64_t M, int64_t num_classes, float* loss,
+                     float* dlogits, void* stream);
+int dtc_sgd_update(float* param, const float* grad, int64_t n, float lr, void* stream);
 
 /* ------------------------------------------------------------ Selector (NEXT-4, diagnostic)
  * Simulation-based Selector, §4.5.2, Eq. (1), Fig. 10.  HOST, pure

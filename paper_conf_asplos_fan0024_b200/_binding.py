@@ -99,11 +99,16 @@ def lib():
             L.dtc_partition_windows.argtypes = [_vp, _i64, _i32, _vp]
             L.dtc_graphconv.argtypes = [_vp, _vp, _i64, _vp, _i64, _vp, _i32, _vp, _vp, _vp]
             L.dtc_graphconv_launches_per_call.argtypes = []
+            L.dtc_graphconv_backward.argtypes = [_vp, _vp, _vp, _vp, _i64, _i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp,
+                                                 _vp, _vp]
+            L.dtc_softmax_xent.argtypes = [_vp, _vp, _i64, _i64, _vp, _vp, _vp]
+            L.dtc_sgd_update.argtypes = [_vp, _vp, _i64, ctypes.c_float, _vp]
             L.dtc_selector_ar.argtypes = [_vp, _i64, _i32, _i32, _vp, _vp, _vp]
             L.dtc_sched_model.argtypes = [_i32, _i64, P(SchedModel)]
             L.dtc_selector_plan.argtypes = [_vp, _i64, P(SchedModel), _vp, _i32, _i32, _vp, P(_Plan)]
             L.dtc_selector_simulate.argtypes = [_vp, _i64, P(SchedModel), P(ctypes.c_double)]
             L.dtc_tca_reorder.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp]
+            L.dtc_tca_reorder_checked.argtypes = [_i64, _i64, _vp, _vp, _i32, _vp, _vp, _vp, _vp]
             L.dtc_nccl_unique_id.argtypes = [_vp]
             L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
             L.dtc_dist_query.argtypes = [_vp, P(_i64), P(_i64), P(_vp)]
@@ -329,6 +334,27 @@ class Format:
                                    _dptr(AH), _dptr(Y), _stream_ptr(stream)), "dtc_graphconv")
         return Y, AH
 
+    def graphconv_backward(self, AH, W, Y, dY, relu=True, At=None, want_dH=True, bias=True, stream=None):
+        """Backward of graphconv (dtc_graphconv_backward): returns dict dW, db (or None), dAH, dH (or None).
+        At: the Format of A^T (Format.build(..., transpose=True)), needed for dH."""
+        import torch
+        M, F_in = AH.shape
+        F_out = W.shape[1]
+        for name, t, shape in (("AH", AH, (self.M, None)), ("W", W, (F_in, None)), ("Y", Y, (self.M, F_out)),
+                               ("dY", dY, (self.M, F_out))):
+            _dense(t, name, shape, torch.float32)
+        dev = AH.device
+        out = {"dZ": torch.empty((self.M, F_out), dtype=torch.float32, device=dev),
+               "dW": torch.empty((F_in, F_out), dtype=torch.float32, device=dev),
+               "db": torch.empty((F_out,), dtype=torch.float32, device=dev) if bias else None,
+               "dAH": torch.empty((self.M, F_in), dtype=torch.float32, device=dev),
+               "dH": torch.empty((self.K, F_in), dtype=torch.float32, device=dev) if want_dH else None}
+        _check(lib().dtc_graphconv_backward(self._h, At.handle if At is not None else None, _dptr(AH), _dptr(W),
+                                            F_in, F_out, 1 if relu else 0, _dptr(Y), _dptr(dY), _dptr(out["dZ"]),
+                                            _dptr(out["dW"]), _dptr(out["db"]), _dptr(out["dAH"]), _dptr(out["dH"]),
+                                            _stream_ptr(stream)), "dtc_graphconv_backward")
+        return out
+
     def spmm_raw(self, B_ptr: int, N: int, ldb: int, C_ptr: int, ldc: int, stream=None):
         _check(lib().dtc_spmm(self._h, B_ptr, N, ldb, C_ptr, ldc, _stream_ptr(stream)), "dtc_spmm")
 
@@ -410,6 +436,64 @@ def selector_ar(rwo, num_sms: int = 148, occupancy: int = 6) -> dict:
             "num_sms": num_sms, "occupancy": occupancy}
 
 
+def softmax_xent(logits, labels, stream=None):
+    """(loss as a 1-element CUDA tensor, dlogits) of the mean softmax cross-entropy (dtc_softmax_xent)."""
+    import torch
+    _dense(logits, "logits", (None, None), torch.float32)
+    if labels.dtype != torch.int32 or not labels.is_cuda or labels.numel() != logits.shape[0]:
+        raise TypeError("labels must be a CUDA int32 tensor with one entry per row")
+    loss = torch.empty((1,), dtype=torch.float32, device=logits.device)
+    dz = torch.empty_like(logits)
+    _check(lib().dtc_softmax_xent(_dptr(logits), _dptr(labels), logits.shape[0], logits.shape[1], _dptr(loss),
+                                  _dptr(dz), _stream_ptr(stream)), "dtc_softmax_xent")
+    return loss, dz
+
+
+def sgd_update(param, grad, lr: float, stream=None):
+    """param -= lr * grad (dtc_sgd_update), in place."""
+    import torch
+    if param.dtype != torch.float32 or grad.dtype != torch.float32 or param.numel() != grad.numel() \
+            or not param.is_contiguous() or not grad.is_contiguous():
+        raise TypeError("param and grad must be contiguous fp32 tensors of equal size")
+    _check(lib().dtc_sgd_update(_dptr(param), _dptr(grad), param.numel(), float(lr), _stream_ptr(stream)),
+           "dtc_sgd_update")
+
+
+class GCN2:
+    """Two GraphConv layers (Eq. (2)) trained with softmax cross-entropy and SGD, every
+    step through the library: H1 = ReLU((A X) W1 + b1), Z = (A H1) W2 + b2, loss = xent(Z, labels);
+    backward dtc_graphconv_backward x 2 (the second needs A^T for dH1), dtc_sgd_update x 4.  This
+    class only sequences C ABI calls (no arithmetic here)."""
+
+    def __init__(self, A, At, F_in: int, F_hid: int, n_classes: int, seed: int = 0):
+        import torch
+        if A.dtype != "tf32" or At.dtype != "tf32" or At.M != A.K or At.K != A.M:
+            raise ValueError("GCN2 needs a TF32 handle of A and of A^T")
+        dev = torch.device("cuda", A.device)
+        g = torch.Generator(device=dev).manual_seed(seed)
+        s1, s2 = (6.0 / (F_in + F_hid)) ** 0.5, (6.0 / (F_hid + n_classes)) ** 0.5
+        self.A, self.At = A, At
+        self.W1 = torch.empty((F_in, F_hid), device=dev).uniform_(-s1, s1, generator=g)
+        self.b1 = torch.zeros((F_hid,), device=dev)
+        self.W2 = torch.empty((F_hid, n_classes), device=dev).uniform_(-s2, s2, generator=g)
+        self.b2 = torch.zeros((n_classes,), device=dev)
+
+    def forward(self, X):
+        Y1, AH1 = self.A.graphconv(X, self.W1, self.b1, relu=True)
+        Z, AH2 = self.A.graphconv(Y1, self.W2, self.b2, relu=False)
+        return Z, (Y1, AH1, AH2)
+
+    def train_step(self, X, labels, lr: float):
+        """One SGD step; returns the loss (1-element CUDA tensor, computed before the update)."""
+        Z, (Y1, AH1, AH2) = self.forward(X)
+        loss, dZ = softmax_xent(Z, labels)
+        g2 = self.A.graphconv_backward(AH2, self.W2, Z, dZ, relu=False, At=self.At, want_dH=True)
+        g1 = self.A.graphconv_backward(AH1, self.W1, Y1, g2["dH"], relu=True, want_dH=False)
+        for p, gr in ((self.W2, g2["dW"]), (self.b2, g2["db"]), (self.W1, g1["dW"]), (self.b1, g1["db"])):
+            sgd_update(p, gr, lr)
+        return loss
+
+
 def sched_model(dtype="tf32", N: int = 128) -> SchedModel:
     """The default B200 launch model for dtype and N on the current device (dtc_sched_model)."""
     m = SchedModel()
@@ -462,6 +546,19 @@ def tca_reorder(M: int, K: int, rowptr, colidx, sm_num: int = 148) -> np.ndarray
     _check(lib().dtc_tca_reorder(M, K, rowptr.ctypes.data_as(_vp), colidx.ctypes.data_as(_vp), sm_num,
                                  perm.ctypes.data_as(_vp)), "dtc_tca_reorder")
     return perm[:M]
+
+
+def tca_reorder_checked(M: int, K: int, rowptr, colidx, sm_num: int = 148):
+    """TCA reordering kept only when it lowers NumTCBlock (dtc_tca_reorder_checked):
+    returns (perm, {"T_identity", "T_reordered", "applied"})."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int32)
+    colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+    perm = np.zeros(max(M, 1), dtype=np.int32)
+    t0, t1, ap = _i64(), _i64(), _i32()
+    _check(lib().dtc_tca_reorder_checked(M, K, rowptr.ctypes.data_as(_vp), colidx.ctypes.data_as(_vp), sm_num,
+                                         perm.ctypes.data_as(_vp), ctypes.byref(t0), ctypes.byref(t1),
+                                         ctypes.byref(ap)), "dtc_tca_reorder_checked")
+    return perm[:M], {"T_identity": t0.value, "T_reordered": t1.value, "applied": bool(ap.value)}
 
 
 def nccl_unique_id() -> bytes:

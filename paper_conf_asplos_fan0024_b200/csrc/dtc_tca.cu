@@ -21,6 +21,7 @@
 #include <cstdint>
 #include <cstring>
 #include <numeric>
+#include <thread>
 #include <vector>
 
 #include "dtc_internal.h"
@@ -187,6 +188,56 @@ extern "C" int dtc_tca_reorder(int64_t M, int64_t K, const int32_t* rowptr, cons
         if (pos != M) { set_error("internal: permutation incomplete"); return DTC_ERR_INVALID; }
     } catch (const std::bad_alloc&) {
         set_error("host OOM in dtc_tca_reorder");
+        return DTC_ERR_OOM;
+    }
+    return DTC_OK;
+}
+
+// NumTCBlock of the matrix with rows in `perm` order (NULL = identity): sum over 16-row windows of
+// ceil(|unique columns| / 8), host threads over windows.
+static int64_t count_tc_blocks(int64_t M, const int32_t* rowptr, const int32_t* colidx, const int32_t* perm) {
+    const int64_t W = (M + kWindow - 1) / kWindow;
+    const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+    std::vector<int64_t> part(nt, 0);
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < nt; ++t)
+        th.emplace_back([&, t]() {
+            std::vector<int32_t> u;
+            int64_t acc = 0;
+            for (int64_t w = t; w < W; w += nt) {
+                u.clear();
+                for (int64_t r = w * kWindow; r < std::min(M, (w + 1) * kWindow); ++r) {
+                    const int64_t row = perm ? perm[r] : r;
+                    u.insert(u.end(), colidx + rowptr[row], colidx + rowptr[row + 1]);
+                }
+                std::sort(u.begin(), u.end());
+                const int64_t nu = std::unique(u.begin(), u.end()) - u.begin();
+                acc += (nu + kTcw - 1) / kTcw;
+            }
+            part[t] = acc;
+        });
+    for (auto& x : th) x.join();
+    int64_t T = 0;
+    for (int64_t v : part) T += v;
+    return T;
+}
+
+extern "C" int dtc_tca_reorder_checked(int64_t M, int64_t K, const int32_t* rowptr, const int32_t* colidx,
+                                       int32_t sm_num, int32_t* perm, int64_t* T_identity, int64_t* T_reordered,
+                                       int32_t* applied) {
+    const int rc = dtc_tca_reorder(M, K, rowptr, colidx, sm_num, perm);
+    if (rc != DTC_OK) return rc;
+    try {
+        const int64_t t0 = count_tc_blocks(M, rowptr, colidx, nullptr);
+        const int64_t t1 = count_tc_blocks(M, rowptr, colidx, perm);
+        const bool use = t1 < t0;
+        if (!use)
+            for (int64_t i = 0; i < M; ++i) perm[i] = (int32_t)i;
+        if (T_identity) *T_identity = t0;
+        if (T_reordered) *T_reordered = t1;
+        if (applied) *applied = use ? 1 : 0;
+    } catch (const std::exception&) {
+        set_error("host failure in dtc_tca_reorder_checked");
         return DTC_ERR_OOM;
     }
     return DTC_OK;

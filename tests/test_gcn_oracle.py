@@ -81,3 +81,85 @@ def test_relu_sign_pattern_and_bound():
     assert np.all(np.abs(Z - b[None, :].astype(np.float64)) <= Bound + 1e-12)
     rtol, atol = ogcn.tolerance("tf32", W)
     assert rtol == pytest.approx(4e-3) and atol.shape == (1, 8)
+
+
+# ------------------------------------------------------------------ backward pins (finite differences)
+def _tiny(seed, M=9, K=11, Fi=3, Fo=2, density=0.35):
+    rng = np.random.default_rng(seed)
+    Ad = (rng.random((M, K)) < density) * rng.uniform(-1, 1, (M, K))
+    rp = np.concatenate([[0], np.cumsum((Ad != 0).sum(1))]).astype(np.int32)
+    ci = np.nonzero(Ad)[1].astype(np.int32)
+    v = Ad[Ad != 0].astype(np.float32)
+    H = rng.uniform(-1, 1, (K, Fi)).astype(np.float32)
+    W = rng.uniform(-1, 1, (Fi, Fo))
+    b = rng.uniform(-1, 1, Fo)
+    R = rng.uniform(-1, 1, (M, Fo))
+    return Ad.astype(np.float32).astype(np.float64), rp, ci, v, H, W, b, R
+
+
+def _loss(Ad, H, W, b, R, relu):
+    Z = Ad @ H.astype(np.float64) @ W + b
+    Y = np.maximum(Z, 0) if relu else Z
+    return float((Y * R).sum()), Y
+
+
+@pytest.mark.parametrize("relu", [False, True])
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_backward_matches_finite_differences(seed, relu):
+    """L = sum(Y * R) so dY = R; every gradient the oracle returns equals the central difference of
+    the FORWARD (a dense FP64 expression, independent of the backward formulas) -- a dropped term,
+    a transposed operand or a wrong sign in dW, db, dH fails."""
+    Ad, rp, ci, v, H, W, b, R = _tiny(seed)
+    M, K = Ad.shape
+    _, Y = _loss(Ad, H, W, b, R, relu)
+    mask = (Y > 0).astype(np.float64) if relu else None
+    g = ogcn.graphconv_backward(M, K, rp, ci, v, H, W, R, mask=mask)
+    eps = 1e-6
+    for (i, j) in [(0, 0), (1, 1), (2, 0)]:
+        Wp, Wm = W.copy(), W.copy()
+        Wp[i, j] += eps
+        Wm[i, j] -= eps
+        fd = (_loss(Ad, H, Wp, b, R, relu)[0] - _loss(Ad, H, Wm, b, R, relu)[0]) / (2 * eps)
+        assert g["dW"][i, j] == pytest.approx(fd, rel=1e-6, abs=1e-7)
+    for j in range(W.shape[1]):
+        bp, bm = b.copy(), b.copy()
+        bp[j] += eps
+        bm[j] -= eps
+        fd = (_loss(Ad, H, W, bp, R, relu)[0] - _loss(Ad, H, W, bm, R, relu)[0]) / (2 * eps)
+        assert g["db"][j] == pytest.approx(fd, rel=1e-6, abs=1e-7)
+    for (k, f) in [(0, 0), (4, 2), (10, 1)]:
+        Hp, Hm = H.astype(np.float64), H.astype(np.float64).copy()
+        Hp = Hp.copy()
+        Hp[k, f] += eps
+        Hm[k, f] -= eps
+        fd = (_loss(Ad, Hp, W, b, R, relu)[0] - _loss(Ad, Hm, W, b, R, relu)[0]) / (2 * eps)
+        assert g["dH"][k, f] == pytest.approx(fd, rel=1e-5, abs=1e-6)
+
+
+def test_csr_transpose_is_dense_transpose():
+    Ad, rp, ci, v, *_ = _tiny(7, M=13, K=6)
+    rp_t, ci_t, v_t = ogcn.csr_transpose(13, 6, rp, ci, v)
+    D = np.zeros((6, 13))
+    for r in range(6):
+        for p in range(rp_t[r], rp_t[r + 1]):
+            D[r, ci_t[p]] = v_t[p]
+        assert np.all(np.diff(ci_t[rp_t[r]:rp_t[r + 1]]) > 0)   # canonical: ascending original row
+    assert np.array_equal(D, Ad.T)
+
+
+def test_softmax_xent_closed_forms_and_fd():
+    C = 7
+    loss, g = ogcn.softmax_xent(np.zeros((5, C)), np.arange(5) % C)
+    assert loss == pytest.approx(np.log(C))
+    assert np.allclose(g.sum(axis=1), 0.0)
+    rng = np.random.default_rng(4)
+    z = rng.normal(size=(4, C))
+    lab = rng.integers(0, C, 4)
+    _, g = ogcn.softmax_xent(z, lab)
+    eps = 1e-6
+    for (i, j) in [(0, 0), (2, 5), (3, int(lab[3]))]:
+        zp, zm = z.copy(), z.copy()
+        zp[i, j] += eps
+        zm[i, j] -= eps
+        fd = (ogcn.softmax_xent(zp, lab)[0] - ogcn.softmax_xent(zm, lab)[0]) / (2 * eps)
+        assert g[i, j] == pytest.approx(fd, rel=1e-6, abs=1e-9)

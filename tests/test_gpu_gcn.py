@@ -99,3 +99,114 @@ def test_graphconv_rejects_bad_arguments():
         f.graphconv(H.half(), torch.zeros((8, 4), device="cuda"))
     from paper_conf_asplos_fan0024_b200 import lib
     assert lib().dtc_graphconv(f.handle, H.data_ptr(), 8, 0, 4, 0, 1, 0, 0, 0) != 0
+
+
+# ------------------------------------------------------------------ backward / training (NEXT-3)
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("name", ["c1", "c2"])
+def test_transposed_format_bit_exact(name, dtype):
+    """opts.transpose: the GPU condenses A^T from A's CSR; bit-exact against O2 of the oracle's
+    CSR transpose (rows of A^T ascending in the original row)."""
+    from gpu_util import assert_format_equal, check_units
+    import oracle
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    v = v.astype(np.float16) if dtype == "fp16" else v
+    ft = build(cfg.M, cfg.K, rp, ci, v, dtype=dtype, transpose=True)
+    assert (ft.M, ft.K, ft.nnz) == (cfg.K, cfg.M, len(ci))
+    rp_t, ci_t, v_t = ogcn.csr_transpose(cfg.M, cfg.K, rp, ci, v)
+    got = ft.export()
+    assert_format_equal(got, oracle.condense(cfg.K, rp_t, ci_t, v_t))
+    check_units(got, cfg.K)
+
+
+def test_transposed_nonsquare_and_empty():
+    import oracle
+    from gpu_util import assert_format_equal
+    M, K = 70, 45
+    rp, ci = datagen.random_csr(M, K, 0.08, 5)
+    v = datagen.uniform(5, 1, len(ci))
+    ft = build(M, K, rp, ci, v, transpose=True)
+    rp_t, ci_t, v_t = ogcn.csr_transpose(M, K, rp, ci, v)
+    assert_format_equal(ft.export(), oracle.condense(K, rp_t, ci_t, v_t))
+    B = datagen.uniform(5, 2, M * 24).reshape(M, 24)
+    from gpu_util import spmm, check_tol
+    check_tol(spmm(ft, B), K, M, rp_t, ci_t, v_t, B, "tf32")
+    f0 = build(M, K, np.zeros(M + 1, np.int32), np.zeros(0, np.int32), np.zeros(0, np.float32), transpose=True)
+    assert (f0.M, f0.num_tc_blocks) == (K, 0)
+
+
+def _bw_check(got, ref, bound, rtol, atol=1e-6, what=""):
+    err = np.abs(got.astype(np.float64) - ref)
+    lim = rtol * bound + atol
+    assert np.all(np.isfinite(got)), what
+    assert np.all(err <= lim), f"{what}: max err/limit {float(np.max(err / lim)):.3g}"
+
+
+@pytest.mark.parametrize("relu", [True, False])
+@pytest.mark.parametrize("name,Fi,Fo", [("c1", 64, 16), ("c1", 33, 7), ("c2", 128, 64)])
+def test_graphconv_backward_vs_oracle(name, Fi, Fo, relu):
+    """dtc_graphconv_backward (dW, db, dAH, dH = A^T dAH on the transposed ME-TCF) against the FP64
+    chain rule; the ReLU mask is the GPU forward's (both sides take the same sign decision)."""
+    import torch
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    H = datagen.uniform(cfg.seed_b, 21, cfg.K * Fi).reshape(cfg.K, Fi)
+    W = datagen.uniform(cfg.seed_b, 22, Fi * Fo).reshape(Fi, Fo) * np.float32(1.0 / np.sqrt(Fi))
+    b = datagen.uniform(cfg.seed_b, 23, Fo)
+    dY = datagen.uniform(cfg.seed_b, 24, cfg.M * Fo).reshape(cfg.M, Fo)
+    f = build(cfg.M, cfg.K, rp, ci, v)
+    ft = build(cfg.M, cfg.K, rp, ci, v, transpose=True)
+    Y, AH = f.graphconv(dev(H), dev(W), dev(b), relu=relu)
+    g = f.graphconv_backward(AH, dev(W), Y, dev(dY), relu=relu, At=ft)
+    torch.cuda.synchronize()
+    Yh = Y.cpu().numpy()
+    mask = (Yh > 0).astype(np.float64) if relu else None
+    ref = ogcn.graphconv_backward(cfg.M, cfg.K, rp, ci, v, H, W, dY, mask=mask)
+    tol = ogcn.backward_tolerance("tf32", cfg.M)
+    _bw_check(g["dW"].cpu().numpy(), ref["dW"], ref["bound_dW"], tol["dW"], what="dW")
+    _bw_check(g["db"].cpu().numpy(), ref["db"], ref["bound_db"], tol["db"], what="db")
+    _bw_check(g["dAH"].cpu().numpy(), ref["dAH"], ref["bound_dAH"], tol["dAH"], what="dAH")
+    _bw_check(g["dH"].cpu().numpy(), ref["dH"], ref["bound_dH"], tol["dH"], what="dH")
+
+
+def test_softmax_xent_vs_oracle():
+    import torch
+    from paper_conf_asplos_fan0024_b200 import softmax_xent, DtcError
+    M, C = 3000, 10
+    z = datagen.uniform(3, 1, M * C).reshape(M, C) * np.float32(4.0)
+    lab = (np.arange(M) * 7 % C).astype(np.int32)
+    loss, dz = softmax_xent(dev(z), dev(lab))
+    torch.cuda.synchronize()
+    rl, rg = ogcn.softmax_xent(z, lab)
+    assert abs(float(loss.item()) - rl) <= 1e-5 * max(1.0, abs(rl))
+    assert np.allclose(dz.cpu().numpy(), rg, rtol=1e-5, atol=1e-8)
+    with pytest.raises(DtcError):
+        softmax_xent(dev(z), dev(np.full(M, C, np.int32)))
+
+
+def test_gcn2_training_reduces_loss():
+    """Two-layer GCN trained for a few SGD steps through the library (forward: dtc_graphconv x 2,
+    loss: dtc_softmax_xent, backward: dtc_graphconv_backward x 2 with A^T, update: dtc_sgd_update);
+    labels are a learnable function of (A X), so the loss must fall."""
+    import torch
+    from paper_conf_asplos_fan0024_b200 import GCN2
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    F0, F1, C = 32, 64, 7
+    X = datagen.uniform(31, 1, cfg.K * F0).reshape(cfg.K, F0)
+    import oracle
+    AX = oracle.spmm(cfg.M, cfg.K, rp, ci, v, X, bound=False)
+    Wt = datagen.uniform(31, 2, F0 * C).reshape(F0, C)
+    labels = np.argmax(AX @ Wt, axis=1).astype(np.int32)
+    A = build(cfg.M, cfg.K, rp, ci, v)
+    At = build(cfg.M, cfg.K, rp, ci, v, transpose=True)
+    net = GCN2(A, At, F0, F1, C, seed=1)
+    Xd, Ld = dev(X), dev(labels)
+    losses = [float(net.train_step(Xd, Ld, lr=1.0).item()) for _ in range(40)]
+    assert all(np.isfinite(losses))
+    assert losses[-1] < 0.9 * losses[0], losses[::8]
+    assert sum(b > a for a, b in zip(losses, losses[1:])) <= 4, losses   # (near-)monotone descent

@@ -87,3 +87,44 @@ def test_tca_raises_mean_nnz_tc_on_shuffled_graph():
     prp, pci = _permute(srp, sci, perm)
     _, T_tca = oracle.condense_count(cfg.M, prp, pci)
     assert T_tca < 0.8 * T_shuf
+
+
+def _permuted(rp, ci, perm):
+    rows = [ci[rp[r]:rp[r + 1]] for r in perm]
+    rp2 = np.concatenate([[0], np.cumsum([len(x) for x in rows])]).astype(np.int32)
+    return rp2, (np.concatenate(rows) if rows else np.zeros(0, np.int32)).astype(np.int32)
+
+
+@pytest.mark.parametrize("name", ["c1", "c4small", "shuffled"])
+def test_tca_checked_keeps_identity_unless_T_drops(name):
+    """dtc_tca_reorder_checked: the T counts equal O2's NumTCBlock (oracle.condense_count) of the two
+    row orders, and the TCA order is applied exactly when it lowers T (else the identity)."""
+    import oracle
+    if name == "c1":
+        cfg = configs.get("c1")
+        rp, ci = configs.make_pattern(cfg)
+        M, K = cfg.M, cfg.K
+    elif name == "c4small":   # banded: already in its best order, TCA cannot lower T
+        M = K = 4000
+        rows = [sorted(set(range(max(0, i - 3), min(K, i + 4)))) for i in range(M)]
+        rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int32)
+        ci = np.concatenate(rows).astype(np.int32)
+    else:                     # shuffled block diagonal (16-row blocks of 8 columns): TCA restores them
+        nb = 64
+        rows = [list(range(8 * (i // 16), 8 * (i // 16) + 8)) for i in range(16 * nb)]
+        rp0 = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int32)
+        ci0 = np.concatenate(rows).astype(np.int32)
+        M, K = 16 * nb, 8 * nb
+        rp, ci = _shuffle_rows(M, rp0, ci0, 5)
+    perm, info = dtc.tca_reorder_checked(M, K, rp, ci, 148)
+    raw = dtc.tca_reorder(M, K, rp, ci, 148)
+    _, t0 = oracle.condense_count(M, rp, ci)
+    rpp, cip = _permuted(rp, ci, raw)
+    _, t1 = oracle.condense_count(M, rpp, cip)
+    assert (info["T_identity"], info["T_reordered"]) == (t0, t1)
+    assert info["applied"] == (t1 < t0)
+    assert np.array_equal(perm, raw if t1 < t0 else np.arange(M, dtype=np.int32))
+    if name == "c4small":
+        assert not info["applied"]
+    if name == "shuffled":
+        assert info["applied"]
