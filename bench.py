@@ -66,6 +66,8 @@ def parse_args():
     p.add_argument("--unit-blocks", type=int, default=0)
     p.add_argument("--guided", type=int, default=0, help="F4 guided tail (1 on, -1 off, 0 auto)")
     p.add_argument("--persistent", type=int, default=0, help="DTC_OPT_PERSISTENT for the timed launches")
+    p.add_argument("--window-rows", type=int, default=0,
+                   help="32: NEXT-2 tall windows (TF32 workloads; FP16 legs keep 16-row ME-TCF)")
     p.add_argument("--selector", type=int, default=0,
                    help="F4 cut by the B200 Selector's plan for this N (NEXT-4, dtc_selector_plan): 1 on, 0 fixed rule")
     p.add_argument("--ncu", default="auto", choices=["auto", "off"],
@@ -348,7 +350,8 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
         torch.cuda.synchronize()
         tb0 = time.perf_counter()
         fmt = dtc.Format.build(rp_d, ci_d, v_d, M, K, dtype=cfg.dtype, unit_blocks=args.unit_blocks,
-                               guided=args.guided, n_hint=N, selector=args.selector)
+                               guided=args.guided, n_hint=N, selector=args.selector,
+                               window_rows=args.window_rows if cfg.dtype == "tf32" else 0)
         torch.cuda.synchronize()
         build_ms_runs.append((time.perf_counter() - tb0) * 1e3)
     fmt.set_option("persistent", args.persistent)
@@ -372,7 +375,7 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
     leg.update({"num_tc_blocks": T, "mean_nnz_tc": round(nnz / max(T, 1), 3), "sum_u": ab["sum_u"],
                 "unit_blocks": fmt.unit_blocks, "num_units": fmt.num_units,
                 "split_windows": fmt.num_split_windows, "guided": fmt.get_option("guided"),
-                "f4_plan": "selector" if args.selector else "rule",
+                "f4_plan": "selector" if args.selector else "rule", "window_rows": fmt.window_rows,
                 "selector_predicted_ms": round(fmt.get_option("plan_makespan_ns") / 1e6, 4) or None,
                 "format_build_ms": round(build_ms_runs[-1], 3),
                 "format_build_first_call_ms": round(build_ms_runs[0], 3),

@@ -73,6 +73,7 @@ typedef struct {
     int64_t M, K, nnz, num_windows, num_tc_blocks, num_units, num_split_windows;
     int32_t dtype;
     int32_t unit_blocks;
+    int32_t window_rows;   /* 16 (ME-TCF) or 32 (dtc_build_opts_t.window_rows) */
     const int32_t* row_window_offset;
     const int32_t* tc_offset;
     const uint8_t* tc_local_id;
@@ -110,6 +111,11 @@ typedef struct {
      * CSR) -- e.g. the handle for the GCN backward dH = A^T dAH (NEXT-3).  Not combinable with
      * row_perm (INVALID). */
     int32_t transpose;
+    /* window_rows = 32: condense with 32-row windows (TC blocks of 32 x 8, local ids 0..255 still in
+     * uint8, SparseAtoB per 32-row window) -- the NEXT-2 layout in which two consecutive 16-row
+     * windows gather their shared B rows once; 0 or 16 = the paper's ME-TCF.  The
+     * view's arrays then describe 32-row windows; dtc_spmm computes the same C. */
+    int32_t window_rows;
 } dtc_build_opts_t;
 
 /* F0-F4: validate CSR, condense into ME-TCF and build the work-unit schedule on

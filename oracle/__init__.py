@@ -62,10 +62,10 @@ def lib():
             L.oracle_spmm.restype = ctypes.c_int
             L.oracle_spmm_at.argtypes = [i64, vp, vp, vp, vp, i64, i64, vp, vp, vp, vp]
             L.oracle_spmm_at.restype = ctypes.c_int
-            L.oracle_condense_count.argtypes = [i64, vp, vp, vp]
-            L.oracle_condense_count.restype = i64
-            L.oracle_condense_fill.argtypes = [i64, vp, vp, vp, i64, vp, vp, vp, vp, vp]
-            L.oracle_condense_fill.restype = ctypes.c_int
+            L.oracle_condense_count_wh.argtypes = [i64, vp, vp, i64, vp]
+            L.oracle_condense_count_wh.restype = i64
+            L.oracle_condense_fill_wh.argtypes = [i64, vp, vp, i64, vp, i64, vp, vp, vp, vp, vp]
+            L.oracle_condense_fill_wh.restype = ctypes.c_int
             L.oracle_max_threads.argtypes = []
             L.oracle_max_threads.restype = ctypes.c_int
             L.oracle_set_threads.argtypes = [ctypes.c_int]
@@ -128,23 +128,24 @@ def spmm_at(M, rowptr, colidx, vals, B, rows, cols):
     return C, Bd
 
 
-def condense_count(M, rowptr, colidx):
-    """O2 steps 1-2: RowWindowOffset and NumTCBlock."""
-    W = (M + WINDOW - 1) // WINDOW
+def condense_count(M, rowptr, colidx, window: int = WINDOW):
+    """O2 steps 1-2: RowWindowOffset and NumTCBlock (window = rows per window: 16, the paper's
+    BLOCK_HEIGHT, or 32 for the NEXT-2 tall windows, reading C2b)."""
+    W = (M + window - 1) // window
     rwo = np.zeros(W + 1, dtype=np.int32)
-    T = lib().oracle_condense_count(M, _p(_c(rowptr, np.int32)), _p(_c(colidx, np.int32)), _p(rwo))
+    T = lib().oracle_condense_count_wh(M, _p(_c(rowptr, np.int32)), _p(_c(colidx, np.int32)), window, _p(rwo))
     if T < 0:
         raise ValueError("NumTCBlock overflows int32")
     return rwo, int(T)
 
 
-def condense(M, rowptr, colidx, vals=None):
+def condense(M, rowptr, colidx, vals=None, window: int = WINDOW):
     """O2: CSR -> ME-TCF arrays (dict).  vals may be float32 or float16 (copied
     bit-for-bit into TCValues), or None (pattern only)."""
     rowptr = _c(rowptr, np.int32)
     colidx = _c(colidx, np.int32)
     nnz = int(rowptr[-1]) if len(rowptr) else 0
-    rwo, T = condense_count(M, rowptr, colidx)
+    rwo, T = condense_count(M, rowptr, colidx, window)
     if vals is None:
         vals = np.zeros(nnz, dtype=np.float32)
     vals = np.ascontiguousarray(vals)
@@ -152,8 +153,8 @@ def condense(M, rowptr, colidx, vals=None):
     lid = np.zeros(max(nnz, 1), dtype=np.uint8)
     atob = np.zeros(max(8 * T, 1), dtype=np.int32)
     tv = np.zeros(max(nnz, 1), dtype=vals.dtype)
-    rc = lib().oracle_condense_fill(M, _p(rowptr), _p(colidx), _p(vals), vals.itemsize, _p(rwo),
-                                    _p(tco), _p(lid), _p(atob), _p(tv))
+    rc = lib().oracle_condense_fill_wh(M, _p(rowptr), _p(colidx), window, _p(vals), vals.itemsize, _p(rwo),
+                                       _p(tco), _p(lid), _p(atob), _p(tv))
     if rc != 0:
         raise RuntimeError("oracle_condense_fill failed")
     return {

@@ -104,10 +104,10 @@ static int cmp_i32(const void* a, const void* b) {
     return (x > y) - (x < y);
 }
 
-/* U = ascending unique column ids of window w's rows; returns |U| (U malloc'd). */
-static int64_t window_unique(int64_t M, const int32_t* rowptr, const int32_t* colidx,
+/* U = ascending unique column ids of window w's rows (windows of wh rows); returns |U| (U malloc'd). */
+static int64_t window_unique(int64_t M, const int32_t* rowptr, const int32_t* colidx, int64_t wh,
                              int64_t w, int32_t** U_out) {
-    int64_t rb = w * WINDOW, re = rb + WINDOW < M ? rb + WINDOW : M;
+    int64_t rb = w * wh, re = rb + wh < M ? rb + wh : M;
     int64_t n = rowptr[re] - rowptr[rb];
     int32_t* U = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     memcpy(U, colidx + rowptr[rb], sizeof(int32_t) * (size_t)n);
@@ -129,15 +129,17 @@ static int64_t rank_of(const int32_t* U, int64_t u, int32_t x) {
     return lo;
 }
 
-/* Steps 1-2: RowWindowOffset[W+1] (int32). Returns NumTCBlock T, or -1. */
-int64_t oracle_condense_count(int64_t M, const int32_t* rowptr, const int32_t* colidx,
-                              int32_t* row_window_offset) {
-    int64_t W = (M + WINDOW - 1) / WINDOW;
+/* Steps 1-2: RowWindowOffset[W+1] (int32). Returns NumTCBlock T, or -1.
+ * wh = rows per window: 16 = the paper's BLOCK_HEIGHT; 32 = the tall windows of the
+ * NEXT-2 layout (reading C2b: the same SGT condensation applied to 32-row windows). */
+int64_t oracle_condense_count_wh(int64_t M, const int32_t* rowptr, const int32_t* colidx, int64_t wh,
+                                 int32_t* row_window_offset) {
+    int64_t W = (M + wh - 1) / wh;
     int64_t* nb = (int64_t*)malloc(sizeof(int64_t) * (size_t)(W > 0 ? W : 1));
     #pragma omp parallel for schedule(dynamic, 16)
     for (int64_t w = 0; w < W; ++w) {
         int32_t* U;
-        int64_t u = window_unique(M, rowptr, colidx, w, &U);
+        int64_t u = window_unique(M, rowptr, colidx, wh, w, &U);
         nb[w] = (u + TCW - 1) / TCW;          /* nTC_w = ceil(u_w / 8) */
         free(U);
     }
@@ -154,18 +156,18 @@ int64_t oracle_condense_count(int64_t M, const int32_t* rowptr, const int32_t* c
 
 /* Steps 3-5: SparseAtoB[8T], TCOffset[T+1], TCLocalId[nnz], TCValues[nnz].
  * vals/tc_values are opaque elements of elem_size bytes (fp32 or fp16). */
-int oracle_condense_fill(int64_t M, const int32_t* rowptr, const int32_t* colidx,
-                         const void* vals, int64_t elem_size, const int32_t* row_window_offset,
-                         int32_t* tc_offset, uint8_t* tc_local_id, int32_t* sparse_a_to_b,
-                         void* tc_values) {
-    int64_t W = (M + WINDOW - 1) / WINDOW;
+int oracle_condense_fill_wh(int64_t M, const int32_t* rowptr, const int32_t* colidx, int64_t wh,
+                            const void* vals, int64_t elem_size, const int32_t* row_window_offset,
+                            int32_t* tc_offset, uint8_t* tc_local_id, int32_t* sparse_a_to_b,
+                            void* tc_values) {
+    int64_t W = (M + wh - 1) / wh;
     const uint8_t* vin = (const uint8_t*)vals;
     uint8_t* vout = (uint8_t*)tc_values;
     int bad = 0;
     #pragma omp parallel for schedule(dynamic, 16) reduction(| : bad)
     for (int64_t w = 0; w < W; ++w) {
         int32_t* U;
-        int64_t u = window_unique(M, rowptr, colidx, w, &U);
+        int64_t u = window_unique(M, rowptr, colidx, wh, w, &U);
         int64_t blk0 = row_window_offset[w];
         int64_t nb = row_window_offset[w + 1] - blk0;
         if (nb != (u + TCW - 1) / TCW) { bad = 1; free(U); continue; }
@@ -176,7 +178,7 @@ int oracle_condense_fill(int64_t M, const int32_t* rowptr, const int32_t* colidx
                 sparse_a_to_b[(blk0 + b) * TCW + i] = k < u ? U[k] : -1;
             }
         /* step 4: traverse the window's nnz in CSR order, bucket by block */
-        int64_t rb = w * WINDOW, re = rb + WINDOW < M ? rb + WINDOW : M;
+        int64_t rb = w * wh, re = rb + wh < M ? rb + wh : M;
         int64_t* cnt = (int64_t*)calloc((size_t)(nb + 1), sizeof(int64_t));
         for (int64_t r = rb; r < re; ++r)
             for (int64_t p = rowptr[r]; p < rowptr[r + 1]; ++p)
@@ -204,4 +206,17 @@ int oracle_condense_fill(int64_t M, const int32_t* rowptr, const int32_t* colidx
     int64_t T = row_window_offset[W];
     tc_offset[T] = rowptr[M];
     return bad ? -1 : 0;
+}
+
+/* The paper's ME-TCF: 16-row windows. */
+int64_t oracle_condense_count(int64_t M, const int32_t* rowptr, const int32_t* colidx,
+                              int32_t* row_window_offset) {
+    return oracle_condense_count_wh(M, rowptr, colidx, WINDOW, row_window_offset);
+}
+int oracle_condense_fill(int64_t M, const int32_t* rowptr, const int32_t* colidx,
+                         const void* vals, int64_t elem_size, const int32_t* row_window_offset,
+                         int32_t* tc_offset, uint8_t* tc_local_id, int32_t* sparse_a_to_b,
+                         void* tc_values) {
+    return oracle_condense_fill_wh(M, rowptr, colidx, WINDOW, vals, elem_size, row_window_offset, tc_offset,
+                                   tc_local_id, sparse_a_to_b, tc_values);
 }

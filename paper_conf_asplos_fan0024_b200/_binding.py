@@ -35,13 +35,15 @@ class _Csr(ctypes.Structure):
 class _View(ctypes.Structure):
     _fields_ = [("M", _i64), ("K", _i64), ("nnz", _i64), ("num_windows", _i64), ("num_tc_blocks", _i64),
                 ("num_units", _i64), ("num_split_windows", _i64), ("dtype", _i32), ("unit_blocks", _i32),
+                ("window_rows", _i32),
                 ("row_window_offset", _vp), ("tc_offset", _vp), ("tc_local_id", _vp),
                 ("sparse_a_to_b", _vp), ("tc_values", _vp), ("units", _vp)]
 
 
 class _Opts(ctypes.Structure):
     _fields_ = [("unit_blocks", _i32), ("dedup_path", _i32), ("guided", _i32), ("window_order", _i32),
-                ("row_perm", _vp), ("n_hint", _i32), ("selector", _i32), ("transpose", _i32)]
+                ("row_perm", _vp), ("n_hint", _i32), ("selector", _i32), ("transpose", _i32),
+                ("window_rows", _i32)]
 
 
 class SchedModel(ctypes.Structure):
@@ -200,6 +202,7 @@ class Format:
         self.num_windows, self.num_tc_blocks = v.num_windows, v.num_tc_blocks
         self.num_units, self.num_split_windows = v.num_units, v.num_split_windows
         self.unit_blocks = v.unit_blocks
+        self.window_rows = v.window_rows
         self.dtype = "fp16" if v.dtype == DTC_FP16 else "tf32"
         self.device = device
         self._trace = None
@@ -208,11 +211,12 @@ class Format:
     def build(cls, rowptr, colidx, vals, M: int, K: int, dtype="tf32", stream=None,
               unit_blocks: int = 0, dedup_path: int = 0, guided: int = 0, row_perm=None,
               window_order: bool = False, n_hint: int = 0, selector: int = 0,
-              transpose: bool = False) -> "Format":
+              transpose: bool = False, window_rows: int = 0) -> "Format":
         """row_perm: optional CUDA int32 tensor [M], new row -> original row (e.g. tca_reorder);
         C is still produced in the original row order.  selector=1 (with unit_blocks=0): F4 cut by
         the B200 Selector's plan for N = n_hint columns (dtc_selector_plan).  transpose=True condenses
-        A^T (K x M) from A's CSR (e.g. for the GCN backward)."""
+        A^T (K x M) from A's CSR (e.g. for the GCN backward).  window_rows=32: the NEXT-2 tall-window
+        layout (two 16-row windows share their gathered B rows; TF32)."""
         csr = _make_csr(rowptr, colidx, vals, M, K, dtype)
         h = ctypes.c_void_p()
         if row_perm is not None:
@@ -220,7 +224,7 @@ class Format:
             if row_perm.dtype != torch.int32 or not row_perm.is_cuda or row_perm.numel() != M:
                 raise TypeError("row_perm must be a CUDA int32 tensor of length M")
         opts = _Opts(int(unit_blocks), int(dedup_path), int(guided), int(bool(window_order)), _dptr(row_perm),
-                     int(n_hint), int(selector), int(bool(transpose)))
+                     int(n_hint), int(selector), int(bool(transpose)), int(window_rows))
         _check(lib().dtc_format_build_ex(ctypes.byref(csr), ctypes.byref(opts), _stream_ptr(stream),
                                          ctypes.byref(h)), "dtc_format_build")
         return cls(h.value, device=rowptr.device.index or 0)

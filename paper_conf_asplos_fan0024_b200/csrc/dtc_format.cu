@@ -45,10 +45,12 @@ __device__ __forceinline__ int64_t clamp64(int64_t v, int64_t lo, int64_t hi) {
     return v < lo ? lo : (v > hi ? hi : v);
 }
 
-// Window w's nnz segment [s0, s1) (clamped so malformed input cannot fault).
+// Window w's nnz segment [s0, s1) (clamped so malformed input cannot fault); windows of WH rows
+// (16 = the paper's BLOCK_HEIGHT; 32 = the tall windows of NEXT-2).
+template <int WH>
 __device__ __forceinline__ void window_segment(const int32_t* rowptr, int64_t M, int64_t nnz, int64_t w,
                                                int64_t* s0, int64_t* s1) {
-    int64_t r0 = w * kWindow, r1 = min(r0 + kWindow, M);
+    int64_t r0 = w * WH, r1 = min(r0 + WH, M);
     int64_t a = clamp64(rowptr[r0], 0, nnz), b = clamp64(rowptr[r1], 0, nnz);
     *s0 = a;
     *s1 = b < a ? a : b;
@@ -84,6 +86,7 @@ __global__ void k_validate(int64_t M, int64_t K, int64_t nnz, const int32_t* __r
 // ---------------------------------------------------------------- F1 (sort path)
 // Output per window: u[w] (unique count), nb[w] = ceil(u/8), uniq[s0 + k] (k < u)
 // ascending unique columns, rank[p] for p in the segment.
+template <int WH>
 __global__ void __launch_bounds__(kSortThreads)
 k_dedup_sort(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowptr,
              const int32_t* __restrict__ colidx, int mode, int32_t* __restrict__ u_out,
@@ -92,7 +95,7 @@ k_dedup_sort(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowp
     __shared__ int s_u[kSortMax];
     const int64_t w = blockIdx.x;
     int64_t s0, s1;
-    window_segment(rowptr, M, nnz, w, &s0, &s1);
+    window_segment<WH>(rowptr, M, nnz, w, &s0, &s1);
     const int64_t n64 = s1 - s0;
     const int n = n64 > INT_MAX ? INT_MAX : (int)n64;
     if (n > kSortMax || mode == 2) return;  // bitmap path handles it
@@ -154,6 +157,7 @@ k_dedup_sort(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowp
 }
 
 // ---------------------------------------------------------------- F1 (bitmap path)
+template <int WH>
 __global__ void __launch_bounds__(kBmThreads)
 k_dedup_bitmap(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ rowptr,
                const int32_t* __restrict__ colidx, int mode, int32_t* __restrict__ u_out,
@@ -163,7 +167,7 @@ k_dedup_bitmap(int64_t M, int64_t K, int64_t nnz, const int32_t* __restrict__ ro
     int* pref = (int*)(smem_bm + kBmWords); // [kBmWords] exclusive popcount prefix
     const int64_t w = blockIdx.x;
     int64_t s0, s1;
-    window_segment(rowptr, M, nnz, w, &s0, &s1);
+    window_segment<WH>(rowptr, M, nnz, w, &s0, &s1);
     const int64_t n = s1 - s0;
     if (mode != 2 && n <= kSortMax) return;  // sort path handled it
     int lo = INT_MAX, hi = -1;
@@ -312,27 +316,28 @@ __global__ void k_to_i32(const int64_t* __restrict__ in, int32_t* __restrict__ o
 constexpr int kFillThreads = 256;
 constexpr int kFillSmemBlocks = 1024;
 
-template <class V>
+template <class V, int WH>
 __global__ void __launch_bounds__(kFillThreads)
 k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ rowptr, const int32_t* __restrict__ rwo,
               const int32_t* __restrict__ u, const int32_t* __restrict__ uniq, const int32_t* __restrict__ rank,
               uint32_t* __restrict__ gmask, const V* __restrict__ vin, int32_t* __restrict__ tco,
               uint8_t* __restrict__ lid, V* __restrict__ vout, int32_t* __restrict__ atob) {
-    __shared__ uint32_t s_mask[kFillSmemBlocks * 4];
+    constexpr int MW = WH * kTcw / 32;   // mask words per block: one bit per local id (128 or 256)
+    __shared__ uint32_t s_mask[kFillSmemBlocks * MW];
     __shared__ int s_off[kFillSmemBlocks];
-    __shared__ int s_rp[kWindow + 1];
+    __shared__ int s_rp[WH + 1];
     const int tid = threadIdx.x;
     const int64_t w = blockIdx.x;
     int64_t s0, s1;
-    window_segment(rowptr, M, nnz, w, &s0, &s1);
-    const int64_t r0 = w * kWindow;
-    const int nrows = (M - r0) < kWindow ? (int)(M - r0) : kWindow;
+    window_segment<WH>(rowptr, M, nnz, w, &s0, &s1);
+    const int64_t r0 = w * WH;
+    const int nrows = (M - r0) < WH ? (int)(M - r0) : WH;
     const int64_t b0 = rwo[w];
     const int nb = (int)(rwo[w + 1] - b0);
     const bool sm = nb <= kFillSmemBlocks;
-    uint32_t* mask = sm ? s_mask : gmask + b0 * 4;
+    uint32_t* mask = sm ? s_mask : gmask + b0 * MW;
     if (tid <= nrows) s_rp[tid] = (int)clamp64(rowptr[r0 + tid], s0, s1);
-    if (sm) for (int i = tid; i < nb * 4; i += kFillThreads) s_mask[i] = 0u;
+    if (sm) for (int i = tid; i < nb * MW; i += kFillThreads) s_mask[i] = 0u;
     const int uw = u[w];
     for (int64_t k = tid; k < (int64_t)nb * kTcw; k += kFillThreads)
         atob[b0 * kTcw + k] = k < uw ? uniq[s0 + k] : -1;
@@ -349,15 +354,17 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
         const int r = row_of(p);
         const int k = rank[p];
         const int id = r * kTcw + (k & 7);
-        atomicOr(&mask[(k >> 3) * 4 + (id >> 5)], 1u << (id & 31));
+        atomicOr(&mask[(k >> 3) * MW + (id >> 5)], 1u << (id & 31));
     }
     __syncthreads();
-    auto mask_word = [&](int j, int q) -> uint32_t { return sm ? s_mask[j * 4 + q] : __ldcg(mask + j * 4 + q); };
+    auto mask_word = [&](int j, int q) -> uint32_t { return sm ? s_mask[j * MW + q] : __ldcg(mask + j * MW + q); };
     int64_t running = s0;
     for (int jb = 0; jb < nb; jb += kFillThreads) {
         const int j = jb + tid;
         int c = 0;
-        if (j < nb) c = __popc(mask_word(j, 0)) + __popc(mask_word(j, 1)) + __popc(mask_word(j, 2)) + __popc(mask_word(j, 3));
+        if (j < nb)
+#pragma unroll
+            for (int q = 0; q < MW; ++q) c += __popc(mask_word(j, q));
         int tot;
         const int ex = block_exscan<kFillThreads>(c, &tot);
         if (j < nb) {
@@ -375,7 +382,7 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
         const int id = r * kTcw + (k & 7);
         int below = 0;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < MW; ++q) {
             const int lo = q * 32;
             const uint32_t m = mask_word(j, q);
             if (id >= lo + 32) below += __popc(m);
@@ -386,7 +393,7 @@ k_fill_window(int64_t W, int64_t M, int64_t nnz, const int32_t* __restrict__ row
         vout[pos] = vin[p];
     }
     if (sm)   // persist the masks (the kernel-side fragment index)
-        for (int i = tid; i < nb * 4; i += kFillThreads) gmask[b0 * 4 + i] = s_mask[i];
+        for (int i = tid; i < nb * MW; i += kFillThreads) gmask[b0 * MW + i] = s_mask[i];
 }
 
 // ---------------------------------------------------------------- F4
@@ -575,11 +582,14 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
     if (transpose && opts->row_perm) { set_error("transpose and row_perm cannot be combined"); return DTC_ERR_INVALID; }
     // the condensed matrix: A (M x K) or A^T (K x M)
     const int64_t Mc = transpose ? K : M, Kc = transpose ? M : K;
-    const int64_t W = (Mc + kWindow - 1) / kWindow;
+    const int WH = (opts && opts->window_rows > 0) ? opts->window_rows : kWindow;
+    if (WH != 16 && WH != 32) { set_error("window_rows must be 16 or 32"); return DTC_ERR_INVALID; }
+    if (WH == 32 && csr->dtype != DTC_TF32) { set_error("window_rows = 32 is implemented for TF32"); return DTC_ERR_UNSUPPORTED; }
+    const int64_t W = (Mc + WH - 1) / WH;
 
     dtc_format* h = new (std::nothrow) dtc_format();
     if (!h) { set_error("host OOM"); return DTC_ERR_OOM; }
-    h->M = Mc; h->K = Kc; h->nnz = nnz; h->W = W; h->dtype = csr->dtype;
+    h->M = Mc; h->K = Kc; h->nnz = nnz; h->W = W; h->dtype = csr->dtype; h->window_h = WH;
     cudaGetDevice(&h->device);
     BuildTemps t;
     dtc_csr_t pcsr;   // permuted CSR view (row_perm)
@@ -687,12 +697,20 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         st.mark("F0 validate");
         // F1
         if (W > 0) {
-            k_dedup_sort<<<(unsigned)W, kSortThreads, 0, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
-                                                             t.u, t.nb, t.uniq, t.rank);
             const size_t bm_smem = 2 * kBmWords * sizeof(uint32_t);
-            TRYC(cudaFuncSetAttribute(k_dedup_bitmap, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
-            k_dedup_bitmap<<<(unsigned)W, kBmThreads, bm_smem, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
-                                                                   t.u, t.nb, t.uniq, t.rank);
+            if (WH == 16) {
+                k_dedup_sort<16><<<(unsigned)W, kSortThreads, 0, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
+                                                                     t.u, t.nb, t.uniq, t.rank);
+                TRYC(cudaFuncSetAttribute(k_dedup_bitmap<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+                k_dedup_bitmap<16><<<(unsigned)W, kBmThreads, bm_smem, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx,
+                                                                           mode, t.u, t.nb, t.uniq, t.rank);
+            } else {
+                k_dedup_sort<32><<<(unsigned)W, kSortThreads, 0, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx, mode,
+                                                                     t.u, t.nb, t.uniq, t.rank);
+                TRYC(cudaFuncSetAttribute(k_dedup_bitmap<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+                k_dedup_bitmap<32><<<(unsigned)W, kBmThreads, bm_smem, s>>>(Mc, Kc, nnz, csr->rowptr, csr->colidx,
+                                                                           mode, t.u, t.nb, t.uniq, t.rank);
+            }
         }
         TRYC(cudaGetLastError());
         st.mark("F1 dedup");
@@ -730,16 +748,19 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         if (T > 0) {
             // occupancy masks: built in shared memory (windows of <= kFillSmemBlocks blocks) or
             // directly in this array, which the SpMM kernel keeps as its fragment index
-            TRY(dalloc(&h->mask, 4 * T, s));
-            TRYC(cudaMemsetAsync(h->mask, 0, 4 * T * sizeof(uint32_t), s));
-            if (h->dtype == DTC_FP16)
-                k_fill_window<uint16_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, Mc, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint16_t*)csr->vals,
-                    h->tco, h->lid, (uint16_t*)h->vals, h->atob);
-            else
-                k_fill_window<uint32_t><<<(unsigned)W, kFillThreads, 0, s>>>(
-                    W, Mc, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, h->mask, (const uint32_t*)csr->vals,
-                    h->tco, h->lid, (uint32_t*)h->vals, h->atob);
+            const int64_t mw = WH * kTcw / 32;   // mask words per block
+            TRY(dalloc(&h->mask, mw * T, s));
+            TRYC(cudaMemsetAsync(h->mask, 0, mw * T * sizeof(uint32_t), s));
+#define DTC_FILL(V, WHV)                                                                                         \
+    k_fill_window<V, WHV><<<(unsigned)W, kFillThreads, 0, s>>>(W, Mc, nnz, csr->rowptr, h->rwo, t.u, t.uniq, t.rank, \
+                                                              h->mask, (const V*)csr->vals, h->tco, h->lid,        \
+                                                              (V*)h->vals, h->atob)
+            if (h->dtype == DTC_FP16) {
+                if (WH == 16) DTC_FILL(uint16_t, 16); else DTC_FILL(uint16_t, 32);
+            } else {
+                if (WH == 16) DTC_FILL(uint32_t, 16); else DTC_FILL(uint32_t, 32);
+            }
+#undef DTC_FILL
         } else {
             TRYC(cudaMemsetAsync(h->tco, 0, sizeof(int32_t), s));
         }
@@ -760,7 +781,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
             TRYC(cudaMemcpyAsync(hrwo.data(), h->rwo, (W + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
             TRYC(cudaStreamSynchronize(s));
             dtc_sched_model_t m;
-            TRY(sched_model(h->dtype, (opts && opts->n_hint > 0) ? opts->n_hint : 128, &m));
+            TRY(sched_model(h->dtype, (opts && opts->n_hint > 0) ? opts->n_hint : 128, &m, WH));
             dtc_plan_t best;
             TRY(selector_plan(hrwo.data(), W, m, nullptr, 0, gopt, nullptr, &best));
             U = best.unit_blocks;
@@ -843,7 +864,7 @@ extern "C" int dtc_format_query(dtc_handle_t h, dtc_format_view_t* v) {
     if (!h || !v) { set_error("null handle or view"); return DTC_ERR_INVALID; }
     v->M = h->M; v->K = h->K; v->nnz = h->nnz; v->num_windows = h->W; v->num_tc_blocks = h->T;
     v->num_units = h->num_units; v->num_split_windows = h->num_split;
-    v->dtype = h->dtype; v->unit_blocks = h->unit_blocks;
+    v->dtype = h->dtype; v->unit_blocks = h->unit_blocks; v->window_rows = h->window_h;
     v->row_window_offset = h->rwo; v->tc_offset = h->tco; v->tc_local_id = h->lid;
     v->sparse_a_to_b = h->atob; v->tc_values = h->vals; v->units = (const int32_t*)h->units;
     return DTC_OK;

@@ -38,6 +38,7 @@ struct Options {
 struct dtc_format {
     int64_t M = 0, K = 0, nnz = 0, W = 0, T = 0;
     int32_t dtype = 0;
+    int32_t window_h = 16;            // rows per window: 16 (ME-TCF) or 32 (tall windows, NEXT-2)
     int32_t unit_blocks = 0;
     int32_t guided = 0;               // F4 guided tail in use
     double plan_makespan_ns = 0.0;    // Selector's simulated makespan of the chosen plan (0 = rule)
@@ -47,10 +48,10 @@ struct dtc_format {
     uint8_t* lid = nullptr;      // [nnz]
     int32_t* atob = nullptr;     // [8T]
     void* vals = nullptr;        // [nnz] fp32 / fp16
-    // kernel-side index derived from TCLocalId (not part of ME-TCF): 128-bit occupancy of each
-    // TC block, bit id = local id.  TCValues[TCOffset[b] + popcount(mask below id)] is the value
+    // kernel-side index derived from TCLocalId (not part of ME-TCF): 128-bit (window_h = 32: 256-bit)
+    // occupancy of each TC block, bit id = local id.  TCValues[TCOffset[b] + popcount(mask below id)] is the value
     // at id (C5: ascending local id), so a lane builds its A fragment without a shared-memory scatter.
-    uint32_t* mask = nullptr;    // [4T]
+    uint32_t* mask = nullptr;    // [4T] (window_h = 32: [8T])
     // F4 schedule
     int64_t num_units = 0;
     int64_t num_split = 0;       // split windows
@@ -146,12 +147,12 @@ struct PadGeometry {
     int64_t cta_cols;
 };
 PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes);
-int pad_occupancy(int dtype, int64_t N);
+int pad_occupancy(int dtype, int64_t N, int window_h = 16);
 
 // B200 Selector (dtc_selector.cu): simulate the F4 units of each candidate plan, return the best
 int selector_plan(const int32_t* rwo, int64_t W, const dtc_sched_model_t& m, const int32_t* cand, int ncand,
                   int guided_opt, dtc_plan_t* plans, dtc_plan_t* best);
-int sched_model(int dtype, int64_t N, dtc_sched_model_t* m);
+int sched_model(int dtype, int64_t N, dtc_sched_model_t* m, int window_h = 16);
 
 // internal build used by the distributed layer: optional row range of the csr
 int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s,

@@ -230,12 +230,12 @@ constexpr double kCtaNs = 2500.0;
 constexpr double kGatherBytesPerNsPerSm = 9296.0 / 148.0;
 constexpr double kFixupNs = 1000.0;
 
-int sched_model(int dtype, int64_t N, dtc_sched_model_t* m) {
+int sched_model(int dtype, int64_t N, dtc_sched_model_t* m, int window_h) {
     if (N < 1) N = 1;
-    const int occ = pad_occupancy(dtype, N);
+    const int occ = pad_occupancy(dtype, N, window_h);
     if (occ < 1) { set_error("cannot query the SpMM kernel occupancy"); return DTC_ERR_CUDA; }
     const PadGeometry g = pad_geometry(dtype, N, 0);
-    const int64_t cols = std::min<int64_t>(N, g.cta_cols);
+    const int64_t cols = std::min<int64_t>(N, window_h == 16 ? g.cta_cols : g.cta_cols / g.slices);
     m->num_sms = num_sms();
     m->occupancy = occ;
     m->cta_ns = kCtaNs;
@@ -250,5 +250,5 @@ extern "C" int dtc_sched_model(int32_t dtype, int64_t N, dtc_sched_model_t* m) {
     if (!m || (dtype != DTC_TF32 && dtype != DTC_FP16)) { set_error("bad sched_model arguments"); return DTC_ERR_INVALID; }
     int n = 0;
     if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) { cudaGetLastError(); set_error("no CUDA device"); return DTC_ERR_CUDA; }
-    return sched_model(dtype, N, m);
+    return sched_model(dtype, N, m, 16);
 }

@@ -259,23 +259,41 @@ __device__ __forceinline__ bool arrive_last(int32_t* ctr, int n, int lane) {
     return last != 0;
 }
 
+// H = 16-row sub-tiles per window (1 for ME-TCF windows, 2 for the 32-row windows of NEXT-2):
+// sub-tile h of split piece slot S is workspace slot S*H + h; one arrival per piece covers all of
+// its sub-tiles.
+template <int H, int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
+__device__ __forceinline__ void split_fixup_h(const Unit& u, float (&acc)[H][NJ][4], float* __restrict__ ws,
+                                              int64_t npad, int32_t* __restrict__ ctr0, int64_t cstride,
+                                              float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int g, int lane,
+                                              int64_t base, int hoff, const int32_t* __restrict__ rowmap) {
+    const int np = u.npieces, G = fixup_group(np);
+    const int g0 = (u.piece / G) * G, gn = min(G, np - g0), ngr = (np + G - 1) / G;
+    const int64_t sb = u.slot_base;
+#pragma unroll
+    for (int h = 0; h < H; ++h) fixup_write<NJ, QPC, CSTRIDE>(acc[h], ws, (sb + u.piece) * H + h, npad, g, base, hoff);
+    if (!arrive_last(ctr0 + (sb + g0) * cstride, gn, lane)) return;
+#pragma unroll
+    for (int h = 0; h < H; ++h) fixup_sum<NJ, QPC, CSTRIDE>(acc[h], ws, (sb + g0) * H + h, H, gn, npad, g, base, hoff);
+    if (ngr > 1) {
+#pragma unroll
+        for (int h = 0; h < H; ++h) fixup_write<NJ, QPC, CSTRIDE>(acc[h], ws, (sb + g0) * H + h, npad, g, base, hoff);
+        if (!arrive_last(ctr0 + (sb + 1) * cstride, ngr, lane)) return;
+#pragma unroll
+        for (int h = 0; h < H; ++h) fixup_sum<NJ, QPC, CSTRIDE>(acc[h], ws, sb * H + h, (int64_t)G * H, ngr, npad, g, base, hoff);
+    }
+#pragma unroll
+    for (int h = 0; h < H; ++h)
+        store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, (int64_t)u.wb * H + h, g, base, hoff, acc[h], false, rowmap);
+}
+
 template <int NJ, bool VEC, int QPC = NJ / 4, int CSTRIDE = 0>
 __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], float* __restrict__ ws, int64_t npad,
                                             int32_t* __restrict__ ctr0, int64_t cstride, float* __restrict__ C,
                                             int64_t ldc, int64_t M, int64_t N, int g, int lane, int64_t base, int hoff,
                                             const int32_t* __restrict__ rowmap) {
-    const int np = u.npieces, G = fixup_group(np);
-    const int g0 = (u.piece / G) * G, gn = min(G, np - g0), ngr = (np + G - 1) / G;
-    const int64_t sb = u.slot_base;
-    fixup_write<NJ, QPC, CSTRIDE>(acc, ws, sb + u.piece, npad, g, base, hoff);
-    if (!arrive_last(ctr0 + (sb + g0) * cstride, gn, lane)) return;
-    fixup_sum<NJ, QPC, CSTRIDE>(acc, ws, sb + g0, 1, gn, npad, g, base, hoff);
-    if (ngr > 1) {
-        fixup_write<NJ, QPC, CSTRIDE>(acc, ws, sb + g0, npad, g, base, hoff);
-        if (!arrive_last(ctr0 + (sb + 1) * cstride, ngr, lane)) return;
-        fixup_sum<NJ, QPC, CSTRIDE>(acc, ws, sb, G, ngr, npad, g, base, hoff);
-    }
-    store_tile<NJ, VEC, QPC, CSTRIDE>(C, ldc, M, N, u.wb, g, base, hoff, acc, false, rowmap);
+    split_fixup_h<1, NJ, VEC, QPC, CSTRIDE>(u, reinterpret_cast<float(&)[1][NJ][4]>(acc), ws, npad, ctr0, cstride, C,
+                                            ldc, M, N, g, lane, base, hoff, rowmap);
 }
 // ============================================================ fallback: register gather
 // 64 zero bytes that padded (-1) B rows and columns beyond N read instead of B
@@ -649,13 +667,31 @@ static_assert(kPadBatch % kFp16PairSpan == 0, "FP16 pairs never straddle an A ba
 // (-1 past the unit), TCOffset[bb], TCOffset[bb + min(kPadBatch, nb)], end of the first window, pad
 constexpr int kFirstRec = kPadBatch * 8 + 4;
 static_assert((kFirstRec * 4) % 16 == 0, "int4 loads of the side record");
-constexpr int kPadAValBytes = kPadBatch * 512 + 128;       // >= batch x 128 values x 4 B + 16, 128-aligned
-constexpr int kPadASlot = kPadAValBytes + kPadBatch * 16;  // + one 16-byte mask per block
-template <int SL, int SEG>
-constexpr size_t pad_smem_bytes() { return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * kPadASlot + 128; }
+// A batch slot for windows of H x 16 rows: values (<= batch x 128H x 4 B + 16, 128-aligned), then
+// one 16H-byte occupancy mask per block
+// (tall windows take batches of kPadBatch / H blocks, so a batch slot is the same size for every H)
+template <int H> constexpr int pad_batch() { return kPadBatch / H; }
+template <int H> constexpr int pad_aval_bytes() { return pad_batch<H>() * 512 * H + 128; }
+template <int H> constexpr int pad_aslot() { return pad_aval_bytes<H>() + pad_batch<H>() * 16 * H; }
+// Cooperative A expansion (consumers decode each block once into shared memory) pays where a
+// CTA has >= 4 consumer warps (each would otherwise decode every block), for FP16 (block pairs),
+// and for tall windows; with 2 TF32 consumer warps its barrier and the 16 KB of fragments (fewer
+// CTAs per SM) cost more than they save: c3 +13.6%, c5 +7.2%, c4/256 +15%, c3h +6.4%, but
+// c2 -14%, c4/128 -13.5% (profiles/r02_ab_coop.txt).
+template <int DT, int SL, int SEG, int H>
+constexpr bool pad_coop() { return DT == DTC_FP16 || SL * SEG / 2 >= 4 || H > 1; }
+template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
+    return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
+}
+template <int SL, int SEG, int H = 1, int DT = DTC_TF32>
+constexpr size_t pad_smem_bytes() {
+    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * pad_aslot<H>() + pad_frag_bytes<DT, SL, SEG, H>() +
+           128;
+}
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
-template <int DT, int SL>
+template <int DT, int SL, int H = 1>
 constexpr int pad_maxregs() {
+    if (H > 1) return SL >= 2 ? 112 : 128;   // two 16-row accumulator tiles per thread
 #ifdef DTC_PAD_MAXREGS
     return DTC_PAD_MAXREGS;
 #else
@@ -696,10 +732,10 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
     return (uint32_t)v;
 }
 
-template <int DT, int SL, int SEG, bool VEC>
+template <int DT, int SL, int SEG, bool VEC, int H>
 // (min-blocks form of the register cap: measured 8-13% faster than __maxnreg__ with the same cap,
 // profiles/r02_ab_launch_bounds.txt)
-__global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL>()))
+__global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL, H>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
@@ -726,9 +762,14 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     constexpr int SLICE_COLS = SEG * COLW1;    // 128 / 256 fp32 or 256 / 512 fp16 columns per slice
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
-    const uint32_t aring = ring + R * STAGE;                          // [2][kPadASlot] A batches
+    constexpr int BATCH = pad_batch<H>();       // TC blocks per A batch
+    constexpr int ASLOT = pad_aslot<H>(), AVAL = pad_aval_bytes<H>();
+    const uint32_t aring = ring + R * STAGE;                          // [2][ASLOT] A batches
     __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[2], bar_aempty[2], bar_ufull[2], bar_uempty[2];
     __shared__ int s_abyte[2];   // byte offset of the batch's first value inside its A slot
+    constexpr bool COOP = pad_coop<DT, SL, SEG, H>();
+    __shared__ uint8_t s_live[2][BATCH];   // COOP: per block, bit h = sub-tile h has a non-zero
+    const uint32_t frags = aring + 2 * ASLOT;  // COOP: [2][BATCH][H] lane-major fragments (expand())
     __shared__ int s_unit[2][10];   // published unit: Unit record, end block of its first window, index (-1 = done)
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -751,7 +792,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&bar_afull[i], 1);
-            mbar_init(&bar_aempty[i], ncons);
+            mbar_init(&bar_aempty[i], COOP ? 1 : ncons);
             mbar_init(&bar_ufull[i], 1);
             mbar_init(&bar_uempty[i], ncons);
         }
@@ -778,7 +819,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             r.e0 = r.e1 = 0;
             if (lane == 0 && i0 < nbu) {
                 r.e0 = __ldg(tco + uu.bb + i0);
-                r.e1 = __ldg(tco + uu.bb + min(i0 + kPadBatch, nbu));
+                r.e1 = __ldg(tco + uu.bb + min(i0 + BATCH, nbu));
             }
             return r;
         };
@@ -846,25 +887,25 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             if (q0 >= num_units) break;
             const int q2 = draw();   // reserve the unit after next now; its latency hides behind this unit
             const int nblocks = u.be - u.bb;
-            for (int i0 = 0; i0 < nblocks; i0 += kPadBatch) {
-                const int c = gc0 + i0 / kPadBatch, aslot = c & 1;
+            for (int i0 = 0; i0 < nblocks; i0 += BATCH) {
+                const int c = gc0 + i0 / BATCH, aslot = c & 1;
                 const BatchMeta cur = finish(rnext);
-                rnext = i0 + kPadBatch < nblocks ? load_raw(u, i0 + kPadBatch) : load_raw(un, 0);
+                rnext = i0 + BATCH < nblocks ? load_raw(u, i0 + BATCH) : load_raw(un, 0);
                 if (i0 == 0) end0n = first_end(un);
-                const int nj = min(kPadBatch, nblocks - i0);
+                const int nj = min(BATCH, nblocks - i0);
                 if (c >= 2) mbar_wait(&bar_aempty[aslot], ((c >> 1) - 1) & 1);
                 if (lane == 0) {
                     const int64_t lo = ((int64_t)cur.e0 * ELT) & ~int64_t(15);
                     const int64_t hi = ((int64_t)cur.e1 * ELT + 15) & ~int64_t(15);
-                    const uint32_t vbytes = (uint32_t)(hi - lo), mbytes = (uint32_t)nj * 16;
-                    const uint32_t dst = aring + aslot * kPadASlot;
+                    const uint32_t vbytes = (uint32_t)(hi - lo), mbytes = (uint32_t)nj * 16 * H;
+                    const uint32_t dst = aring + aslot * ASLOT;
                     s_abyte[aslot] = (int)((int64_t)cur.e0 * ELT - lo);
                     mbar_arrive_tx(&bar_afull[aslot], vbytes + mbytes);
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                                  ::"r"(dst), "l"(reinterpret_cast<const uint8_t*>(avals) + lo), "r"(vbytes),
                                  "r"(smem_u32(&bar_afull[aslot])) : "memory");
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                                 ::"r"(dst + kPadAValBytes), "l"(mask + u.bb + i0), "r"(mbytes),
+                                 ::"r"(dst + AVAL), "l"(mask + (int64_t)(u.bb + i0) * H), "r"(mbytes),
                                  "r"(smem_u32(&bar_afull[aslot])) : "memory");
                 }
                 for (int j = 0; j < nj; ++j) {
@@ -892,7 +933,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 end0n = first_end(un);
             }
             gi0 += nblocks;
-            gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
+            gc0 += (nblocks + BATCH - 1) / BATCH;
             q0 = q1;
             u = un;
             end0 = end0n;
@@ -928,19 +969,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const uint32_t roff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + cg * 16;
     const uint32_t roff1 = roff0 + ODD;
 
-    // A batch cursor: the next block's first value (bytes) and the batch's mask array
-    uint32_t vaddr = 0, maddr = 0;
-    // S1: the A fragment of block i of the unit (batch c = gc0 + i / kPadBatch) from the occupancy
-    // mask and the batch's values (ascending local id, C5); blocks are visited in order
-    auto afrag = [&](int i, int gc0, uint32_t (&a)[FW]) {
-        const int j = i % kPadBatch, c = gc0 + i / kPadBatch;
-        if (j == 0) {
-            mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
-            const uint32_t slot = aring + (c & 1) * kPadASlot;
-            vaddr = slot + s_abyte[c & 1];
-            maddr = slot + kPadAValBytes;
-        }
-        const uint4 m = lds128(maddr + j * 16);
+    // S1, decoding one 16-row sub-tile of a TC block into this lane's mma A fragment: the occupancy
+    // mask m and the block's values at vaddr (ascending local id, C5)
+    auto decode = [&](const uint4 m, uint32_t vaddr, uint32_t (&a)[FW]) {
         const uint32_t wl = upper ? m.y : m.x, wh = upper ? m.w : m.z;
         const int c0 = __popc(m.x), c01 = c0 + __popc(m.y);
         const int rl = (upper ? c0 : 0) + __popc(wl & below);
@@ -956,15 +987,113 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             a[0] = lds16_pred(vaddr + 2 * rl, p00) | (lds16_pred(vaddr + 2 * (rl + p00), p01) << 16);
             a[1] = lds16_pred(vaddr + 2 * rh, p10) | (lds16_pred(vaddr + 2 * (rh + p10), p11) << 16);
         }
-        vaddr += ELT * (c01 + __popc(m.z) + __popc(m.w));
+    };
+    // Cooperative expansion: at the start of batch c the consumer warps decode its blocks ONCE
+    // (warp k takes blocks k, k + ncons, ...) into lane-major fragments in shared memory (FRAG[c&1]),
+    // then every warp reads its fragment with one LDS per sub-tile -- instead of each warp decoding
+    // every block for its own columns (the decode is ~30 instructions per sub-tile).  One named
+    // barrier per batch among the consumers; the raw A slot is released after it, and FRAG[c&1] is
+    // rewritten only at batch c+2, after every consumer has passed the barrier of batch c+1.
+    constexpr int FSUB = 32 * FW * 4;                      // bytes of one sub-tile's fragments
+    auto expand = [&](int c, int nj) {
+        mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
+        const uint32_t slot = aring + (c & 1) * ASLOT;
+        const uint32_t v0 = slot + s_abyte[c & 1], maddr = slot + AVAL;
+        // value offset of every block of the batch: exclusive warp scan of the blocks' popcounts
+        int cnt = 0;
+        if (lane < nj)
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+                const uint4 m = lds128(maddr + (lane * H + h) * 16);
+                cnt += __popc(m.x) + __popc(m.y) + __popc(m.z) + __popc(m.w);
+            }
+        int off = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, off, o);
+            if (lane >= o) off += y;
+        }
+        off -= cnt;
+        const uint32_t fbase = frags + (c & 1) * (BATCH * H * FSUB);
+        for (int jj = warp; jj < nj; jj += ncons) {
+            uint32_t va = v0 + ELT * __shfl_sync(0xffffffffu, off, jj);
+            uint32_t lv = 0;
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+                const uint4 m = lds128(maddr + (jj * H + h) * 16);
+                uint32_t a[FW];
+                decode(m, va, a);
+                va += ELT * (__popc(m.x) + __popc(m.y) + __popc(m.z) + __popc(m.w));
+                lv |= ((m.x | m.y | m.z | m.w) != 0u ? 1u : 0u) << h;
+                const uint32_t dst = fbase + (jj * H + h) * FSUB + lane * FW * 4;
+                if constexpr (FW == 4)
+                    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(a[0]), "r"(a[1]), "r"(a[2]),
+                                 "r"(a[3]) : "memory");
+                else
+                    asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(dst), "r"(a[0]), "r"(a[1]) : "memory");
+            }
+            if (lane == 0) s_live[c & 1][jj] = (uint8_t)lv;
+        }
+        asm volatile("bar.sync 1, %0;" ::"r"(ncons * 32) : "memory");
+        if (warp == 0 && lane == 0) mbar_arrive(&bar_aempty[c & 1]);   // raw values and masks consumed
+    };
+    // this lane's fragments of block i (batch c = gc0 + i / BATCH); live[h] = sub-tile h has a
+    // non-zero (warp-uniform)
+    auto afrag_coop = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
+        const int j = i % BATCH, c = gc0 + i / BATCH;
+        const uint32_t fbase = frags + (c & 1) * (BATCH * H * FSUB) + j * H * FSUB + lane * FW * 4;
+        const uint32_t lv = s_live[c & 1][j];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            live[h] = (lv >> h) & 1u;
+            if constexpr (FW == 4) {
+                const uint4 x = lds128(fbase + h * FSUB);
+                a[h][0] = x.x; a[h][1] = x.y; a[h][2] = x.z; a[h][3] = x.w;
+            } else {
+                const uint2 x = lds64(fbase + h * FSUB);
+                a[h][0] = x.x; a[h][1] = x.y;
+            }
+        }
+    };
+    auto release_coop = [&](int i, int gi, int nblocks, int gc0) {
+        if (lane == 0) mbar_arrive(&bar_empty[gi % R]);
+    };
+
+    // A batch cursor: the next block's first value (bytes) and the batch's mask array
+    uint32_t vaddr = 0, maddr = 0;
+    // S1: the A fragments of block i of the unit (batch c = gc0 + i / BATCH) -- one per 16-row
+    // sub-tile h < H -- decoded by every consumer warp for its own columns; blocks in order
+    auto afrag_dec = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
+        const int j = i % BATCH, c = gc0 + i / BATCH;
+        if (j == 0) {
+            mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
+            const uint32_t slot = aring + (c & 1) * ASLOT;
+            vaddr = slot + s_abyte[c & 1];
+            maddr = slot + AVAL;
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const uint4 m = lds128(maddr + (j * H + h) * 16);
+            live[h] = (m.x | m.y | m.z | m.w) != 0u;
+            decode(m, vaddr, a[h]);
+            vaddr += ELT * (__popc(m.x) + __popc(m.y) + __popc(m.z) + __popc(m.w));
+        }
     };
     // release the B stage of CTA block gi and, after a batch's last block, its A slot
-    auto release = [&](int i, int gi, int nblocks, int gc0) {
+    auto release_dec = [&](int i, int gi, int nblocks, int gc0) {
         if (lane == 0) {
             mbar_arrive(&bar_empty[gi % R]);
-            const int j = i % kPadBatch;
-            if (j == kPadBatch - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[(gc0 + i / kPadBatch) & 1]);
+            const int j = i % BATCH;
+            if (j == BATCH - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) & 1]);
         }
+    };
+    auto afrag = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
+        if constexpr (COOP) afrag_coop(i, gc0, a, live);
+        else afrag_dec(i, gc0, a, live);
+    };
+    auto release = [&](int i, int gi, int nblocks, int gc0) {
+        if constexpr (COOP) release_coop(i, gi, nblocks, gc0);
+        else release_dec(i, gi, nblocks, gc0);
     };
 
     // Units arrive from the producer (s_unit), record and first-window end already loaded, so a
@@ -986,15 +1115,23 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (uidx < 0) break;
         const int nblocks = u.be - u.bb;
         const bool split = u.split_id >= 0;
-        float acc[NJ][4];
+        float acc[H][NJ][4];
 #pragma unroll
-        for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+        for (int h = 0; h < H; ++h)
+#pragma unroll
+            for (int j = 0; j < NJ; ++j) acc[h][j][0] = acc[h][j][1] = acc[h][j][2] = acc[h][j][3] = 0.f;
+        // C rows of window w: the 16-row tiles w*H .. w*H+H-1
+        auto store_window = [&](int w, bool zero) {
+#pragma unroll
+            for (int h = 0; h < H; ++h)
+                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, (int64_t)w * H + h, g, base, hoff, acc[h], zero, rowmap);
+        };
         int cur = u.wb;
         int next_end = INT_MAX;
         if (!split) {
             int e = end0;
             while (cur < u.we && e <= u.bb) {   // leading empty windows
-                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                store_window(cur, true);
                 ++cur;
                 e = cur < u.we ? rwo[cur + 1] : INT_MAX;
             }
@@ -1002,13 +1139,16 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         for (int i = 0; i < nblocks;) {
             const int gi = gi0 + i, s = gi % R;
+            if constexpr (COOP)
+                if (i % BATCH == 0) expand(gc0 + i / BATCH, min(BATCH, nblocks - i));
             // FP16: two TC blocks of one window feed one m16n8k16 (k = block i's 8 columns, then
             // block i+1's -- the k16 A/B fragments are exactly the two k8 fragments side by side)
             const bool pair = fp16_pair(DT, i, nblocks, u.bb, next_end);
-            uint32_t a[FW], a2[FW];
-            afrag(i, gc0, a);
-            if (pair) afrag(i + 1, gc0, a2);
-            // S2/S3: B fragments from the padded stage(s), mma
+            uint32_t a[H][FW], a2[H][FW];
+            bool live[H], live2[H];
+            afrag(i, gc0, a, live);
+            if (pair) afrag(i + 1, gc0, a2, live2);
+            // S2/S3: B fragments from the padded stage(s), mma (a sub-tile without non-zeros is skipped)
             mbar_wait(&bar_full[s], (gi / R) & 1);
             if (tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();
             const uint32_t st = ring + s * STAGE;
@@ -1020,14 +1160,16 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                     const uint32_t y0[4] = {x0.x, x0.y, x0.z, x0.w};
                     const uint32_t y1[4] = {x1.x, x1.y, x1.z, x1.w};
 #pragma unroll
-                    for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[cw * NJ1 + jj], a, y0[jj & 3], y1[jj & 3]);
+                    for (int h = 0; h < H; ++h)
+                        if (H == 1 || live[h])
+#pragma unroll
+                            for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[h][cw * NJ1 + jj], a[h], y0[jj & 3], y1[jj & 3]);
                 }
             } else {
                 if (pair) {
                     const int s2 = (gi + 1) % R;
                     mbar_wait(&bar_full[s2], ((gi + 1) / R) & 1);
                     const uint32_t st2 = ring + s2 * STAGE;
-                    const uint32_t aa[4] = {a[0], a[1], a2[0], a2[1]};
 #pragma unroll
                     for (int cw = 0; cw < CW; ++cw) {
                         const uint4 x0 = lds128(st + roff0 + cw * 128), x1 = lds128(st + roff1 + cw * 128);
@@ -1035,23 +1177,30 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                         const uint32_t y0[4] = {x0.x, x0.y, x0.z, x0.w}, y1[4] = {x1.x, x1.y, x1.z, x1.w};
                         const uint32_t w0[4] = {z0.x, z0.y, z0.z, z0.w}, w1[4] = {z1.x, z1.y, z1.z, z1.w};
 #pragma unroll
-                        for (int jj = 0; jj < NJ1; ++jj) {
-                            const uint32_t sel = (jj & 1) ? 0x7632 : 0x5410;
-                            const uint32_t b0 = __byte_perm(y0[(jj >> 1) & 3], y1[(jj >> 1) & 3], sel);
-                            const uint32_t b1 = __byte_perm(w0[(jj >> 1) & 3], w1[(jj >> 1) & 3], sel);
-                            mma_f16_k16(acc[cw * NJ1 + jj], aa, b0, b1);
+                        for (int h = 0; h < H; ++h) {
+                            const uint32_t aa[4] = {a[h][0], a[h][1], a2[h][0], a2[h][1]};
+#pragma unroll
+                            for (int jj = 0; jj < NJ1; ++jj) {
+                                const uint32_t sel = (jj & 1) ? 0x7632 : 0x5410;
+                                const uint32_t b0 = __byte_perm(y0[(jj >> 1) & 3], y1[(jj >> 1) & 3], sel);
+                                const uint32_t b1 = __byte_perm(w0[(jj >> 1) & 3], w1[(jj >> 1) & 3], sel);
+                                mma_f16_k16(acc[h][cw * NJ1 + jj], aa, b0, b1);
+                            }
                         }
                     }
                 } else {
-                    const uint32_t aa[2] = {a[0], a[1]};
 #pragma unroll
                     for (int cw = 0; cw < CW; ++cw) {
                         const uint4 x0 = lds128(st + roff0 + cw * 128), x1 = lds128(st + roff1 + cw * 128);
                         const uint32_t y0[4] = {x0.x, x0.y, x0.z, x0.w}, y1[4] = {x1.x, x1.y, x1.z, x1.w};
 #pragma unroll
-                        for (int jj = 0; jj < NJ1; ++jj) {
-                            const uint32_t bb = __byte_perm(y0[(jj >> 1) & 3], y1[(jj >> 1) & 3], (jj & 1) ? 0x7632 : 0x5410);
-                            mma_f16(acc[cw * NJ1 + jj], aa, bb);
+                        for (int h = 0; h < H; ++h) {
+                            const uint32_t aa[2] = {a[h][0], a[h][1]};
+#pragma unroll
+                            for (int jj = 0; jj < NJ1; ++jj) {
+                                const uint32_t bb = __byte_perm(y0[(jj >> 1) & 3], y1[(jj >> 1) & 3], (jj & 1) ? 0x7632 : 0x5410);
+                                mma_f16(acc[h][cw * NJ1 + jj], aa, bb);
+                            }
                         }
                     }
                 }
@@ -1062,25 +1211,27 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             i += pair ? 2 : 1;
 
             if (u.bb + i == next_end) {
-                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, false, rowmap);
+                store_window(cur, false);
 #pragma unroll
-                for (int jj = 0; jj < NJ; ++jj) acc[jj][0] = acc[jj][1] = acc[jj][2] = acc[jj][3] = 0.f;
+                for (int h = 0; h < H; ++h)
+#pragma unroll
+                    for (int jj = 0; jj < NJ; ++jj) acc[h][jj][0] = acc[h][jj][1] = acc[h][jj][2] = acc[h][jj][3] = 0.f;
                 ++cur;
                 while (cur < u.we && rwo[cur + 1] == rwo[cur]) {
-                    store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap);
+                    store_window(cur, true);
                     ++cur;
                 }
                 next_end = cur < u.we ? rwo[cur + 1] : INT_MAX;
             }
         }
         if (!split) {
-            while (cur < u.we) { store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, cur, g, base, hoff, acc, true, rowmap); ++cur; }
+            while (cur < u.we) { store_window(cur, true); ++cur; }
         } else {
-            split_fixup<NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp, (int64_t)gridDim.y * 8, C,
-                                             ldc, M, N, g, lane, base, hoff, rowmap);
+            split_fixup_h<H, NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp,
+                                                  (int64_t)gridDim.y * 8, C, ldc, M, N, g, lane, base, hoff, rowmap);
         }
         gi0 += nblocks;
-        gc0 += (nblocks + kPadBatch - 1) / kPadBatch;
+        gc0 += (nblocks + BATCH - 1) / BATCH;
     }
     if (tr && threadIdx.x == 0) tr[5] = gtimer();
 }
@@ -1183,7 +1334,7 @@ static cudaError_t launch_ldg(const LaunchArgs& a, int warps) {
 
 __global__ void k_units_first(int64_t nu, const Unit* __restrict__ units, const int32_t* __restrict__ atob,
                               const int32_t* __restrict__ tco, const int32_t* __restrict__ rwo,
-                              int32_t* __restrict__ out) {
+                              int32_t* __restrict__ out, int batch) {
     for (int64_t q = blockIdx.x; q < nu; q += gridDim.x) {
         const Unit u = units[q];
         const int nb = u.be - u.bb;
@@ -1192,11 +1343,11 @@ __global__ void k_units_first(int64_t nu, const Unit* __restrict__ units, const 
             int32_t v = 0;
             if (t < kPadBatch * 8) {
                 const int i = t / 8;
-                v = i < nb ? atob[(int64_t)(u.bb + i) * 8 + (t % 8)] : -1;
+                v = (i < nb && i < batch) ? atob[(int64_t)(u.bb + i) * 8 + (t % 8)] : -1;
             } else if (t == kPadBatch * 8) {
                 v = nb > 0 ? tco[u.bb] : 0;
             } else if (t == kPadBatch * 8 + 1) {
-                v = nb > 0 ? tco[u.bb + min(kPadBatch, nb)] : 0;
+                v = nb > 0 ? tco[u.bb + min(batch, nb)] : 0;
             } else if (t == kPadBatch * 8 + 2) {
                 v = (u.split_id < 0 && u.wb < u.we) ? rwo[u.wb + 1] : INT_MAX;
             }
@@ -1212,8 +1363,8 @@ static cudaError_t first_records(dtc_format* h, cudaStream_t s) {
     if (h->ufirst || h->num_units == 0) return cudaSuccess;
     int32_t* d = nullptr;
     if (dalloc(&d, (size_t)h->num_units * kFirstRec, s) != DTC_OK) return cudaErrorMemoryAllocation;
-    k_units_first<<<(unsigned)std::min<int64_t>(h->num_units, 65535), 128, 0, s>>>(h->num_units, h->units, h->atob,
-                                                                                  h->tco, h->rwo, d);
+    k_units_first<<<(unsigned)std::min<int64_t>(h->num_units, 65535), 128, 0, s>>>(
+        h->num_units, h->units, h->atob, h->tco, h->rwo, d, h->window_h == kWindow ? pad_batch<1>() : pad_batch<2>());
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { dfree(d, s); return e; }
     h->ufirst = d;
@@ -1240,12 +1391,12 @@ static cudaError_t lpt_units(dtc_format* h, cudaStream_t s) {
     return cudaSuccess;
 }
 
-template <int DT, int SL, int SEG, bool VEC>
+template <int DT, int SL, int SEG, bool VEC, int H>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
-    constexpr size_t smem = pad_smem_bytes<SL, SEG>();
+    constexpr size_t smem = pad_smem_bytes<SL, SEG, H, DT>();
     constexpr int threads = (SL * SEG / 2 + 1) * 32;
     static KernelState ks;
-    const int per_sm = kernel_setup(k_spmm_pad<DT, SL, SEG, VEC>, threads, smem, ks, a.h->device);
+    const int per_sm = kernel_setup(k_spmm_pad<DT, SL, SEG, VEC, H>, threads, smem, ks, a.h->device);
     if (per_sm < 0) {
         const cudaError_t e = cudaGetLastError();
         return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
@@ -1279,16 +1430,22 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     }
     const dim3 grid((unsigned)gx, (unsigned)a.gy);
     int64_t* trace = (h->trace && (int64_t)grid.x * grid.y <= h->trace_cap) ? h->trace : nullptr;
-    k_spmm_pad<DT, SL, SEG, VEC><<<grid, threads, smem, a.s>>>(
+    k_spmm_pad<DT, SL, SEG, VEC, H><<<grid, threads, smem, a.s>>>(
         map, units, h->rwo, h->tco, reinterpret_cast<const uint4*>(h->mask), h->atob, h->vals, a.C, a.ldc, h->M, a.N,
         h->ws, h->counters, a.npad, h->rowmap, trace, (int)h->num_units, uctr, a.te, ufirst);
     return cudaGetLastError();
 }
 
+template <int DT, bool VEC, int H>
+static cudaError_t dispatch_pad_h(int slices, const LaunchArgs& a, const CUtensorMap& map) {
+    if (a.seg == 8) return slices >= 2 ? launch_pad<DT, 2, 8, VEC, H>(a, map) : launch_pad<DT, 1, 8, VEC, H>(a, map);
+    return slices >= 2 ? launch_pad<DT, 2, 4, VEC, H>(a, map) : launch_pad<DT, 1, 4, VEC, H>(a, map);
+}
 template <int DT, bool VEC>
 static cudaError_t dispatch_pad(int slices, const LaunchArgs& a, const CUtensorMap& map) {
-    if (a.seg == 8) return slices >= 2 ? launch_pad<DT, 2, 8, VEC>(a, map) : launch_pad<DT, 1, 8, VEC>(a, map);
-    return slices >= 2 ? launch_pad<DT, 2, 4, VEC>(a, map) : launch_pad<DT, 1, 4, VEC>(a, map);
+    if (DT == DTC_TF32 && a.h->window_h == 32)
+        return a.seg == 8 ? launch_pad<DTC_TF32, 1, 8, VEC, 2>(a, map) : launch_pad<DTC_TF32, 1, 4, VEC, 2>(a, map);
+    return dispatch_pad_h<DT, VEC, 1>(slices, a, map);
 }
 
 // Padded-path geometry for N columns: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB,
@@ -1308,24 +1465,29 @@ PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes) {
 
 // Resident CTAs per SM of the padded kernel dtc_spmm would launch for N columns (vector C path), on
 // the current device -- the measured occupancy the Selector plans with.
-int pad_occupancy(int dtype, int64_t N) {
+int pad_occupancy(int dtype, int64_t N, int window_h) {
     const PadGeometry g = pad_geometry(dtype, N, 0);
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return -1; }
-    auto occ = [&](auto kern, int sl, int seg) -> int {
-        static KernelState ks[8];
-        const int idx = (dtype == DTC_FP16 ? 4 : 0) + (sl - 1) * 2 + (seg == 8 ? 1 : 0);
-        const int threads = (sl * seg / 2 + 1) * 32;
-        const size_t smem = sl == 1 ? (seg == 4 ? pad_smem_bytes<1, 4>() : pad_smem_bytes<1, 8>())
-                                    : (seg == 4 ? pad_smem_bytes<2, 4>() : pad_smem_bytes<2, 8>());
-        return kernel_setup(kern, threads, smem, ks[idx], dev);
+    auto occ = [&](auto kern, int sl, int seg, size_t smem) -> int {
+        static KernelState ks;   // one per kernel instantiation (the lambda is instantiated per kernel type)
+        return kernel_setup(kern, (sl * seg / 2 + 1) * 32, smem, ks, dev);
     };
-    if (dtype == DTC_FP16) {
-        if (g.seg == 8) return g.slices >= 2 ? occ(k_spmm_pad<DTC_FP16, 2, 8, true>, 2, 8) : occ(k_spmm_pad<DTC_FP16, 1, 8, true>, 1, 8);
-        return g.slices >= 2 ? occ(k_spmm_pad<DTC_FP16, 2, 4, true>, 2, 4) : occ(k_spmm_pad<DTC_FP16, 1, 4, true>, 1, 4);
+#define DTC_OCC(DT, H)                                                                                              \
+    do {                                                                                                            \
+        if (g.seg == 8)                                                                                             \
+            return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 8, true, H>, 2, 8, pad_smem_bytes<2, 8, H, DT>())               \
+                                 : occ(k_spmm_pad<DT, 1, 8, true, H>, 1, 8, pad_smem_bytes<1, 8, H, DT>());              \
+        return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 4, true, H>, 2, 4, pad_smem_bytes<2, 4, H, DT>())                   \
+                             : occ(k_spmm_pad<DT, 1, 4, true, H>, 1, 4, pad_smem_bytes<1, 4, H, DT>());                  \
+    } while (0)
+    if (dtype == DTC_FP16) DTC_OCC(DTC_FP16, 1);
+    if (window_h == 32) {   // one slice per CTA (see spmm_launch)
+        if (g.seg == 8) return occ(k_spmm_pad<DTC_TF32, 1, 8, true, 2>, 1, 8, pad_smem_bytes<1, 8, 2>());
+        return occ(k_spmm_pad<DTC_TF32, 1, 4, true, 2>, 1, 4, pad_smem_bytes<1, 4, 2>());
     }
-    if (g.seg == 8) return g.slices >= 2 ? occ(k_spmm_pad<DTC_TF32, 2, 8, true>, 2, 8) : occ(k_spmm_pad<DTC_TF32, 1, 8, true>, 1, 8);
-    return g.slices >= 2 ? occ(k_spmm_pad<DTC_TF32, 2, 4, true>, 2, 4) : occ(k_spmm_pad<DTC_TF32, 1, 4, true>, 1, 4);
+    DTC_OCC(DTC_TF32, 1);
+#undef DTC_OCC
 }
 
 // RAII: make the handle's device current for the duration of a call
@@ -1363,13 +1525,41 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     const PadGeometry pg = pad_geometry(h->dtype, N, h->opt.slice_bytes);
     const int seg = pg.seg;
     const int te = ((N * elt) % 8 == 0) ? 8 : 4;
-    bool pad = h->opt.kernel != 1 && tma_ok && make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg, te);
+    if (h->window_h != kWindow && !tma_ok && h->T > 0) {
+        // tall windows run on the padded kernel only: stage B in a library-owned buffer with a
+        // 16-byte aligned row pitch (a plain strided copy; the arithmetic is unchanged)
+        const int64_t ldb2 = (N + 3) / 4 * 4;
+        const size_t need = (size_t)std::max<int64_t>(h->K, 1) * ldb2 * elt;
+        if (need > h->stage_B_bytes) {
+            dfree(h->stage_B, s);
+            h->stage_B_bytes = 0;
+            uint8_t* sb = nullptr;
+            int rc = dalloc(&sb, need, s);
+            if (rc) return rc;
+            h->stage_B = sb;
+            h->stage_B_bytes = need;
+        }
+        if (h->K > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(h->stage_B, ldb2 * elt, B, ldb * elt, N * elt, h->K, cudaMemcpyDeviceToDevice, s));
+        B = h->stage_B;
+        ldb = ldb2;
+    }
+    const bool tma_ok2 = (h->T > 0) && ((uintptr_t)B % 16 == 0) && ((ldb * elt) % 16 == 0) && ((N * elt) % 4 == 0) &&
+                         h->K < (int64_t(1) << 31) && N < (int64_t(1) << 31);
+    bool pad = (h->opt.kernel != 1 || h->window_h != kWindow) && tma_ok2 &&
+               make_bmap_pad(&map, B, h->K, N, ldb, h->dtype, seg, te);
+    if (!pad && h->window_h != kWindow && h->T > 0) {
+        set_error("tall-window formats need the padded TMA kernel (tensor map encoding failed)");
+        return DTC_ERR_UNSUPPORTED;
+    }
     int64_t cta_cols, slices = 1;
     int warps = 1;
     const int colw_ldg = (h->dtype == DTC_FP16 ? Traits<DTC_FP16>::COLW : Traits<DTC_TF32>::COLW) * kLdgColChunks;
     if (pad) {
-        slices = pg.slices;
-        cta_cols = pg.cta_cols;
+        // tall windows keep one slice per CTA (two accumulator tiles per thread leave no registers for
+        // a second slice; wider B takes more column groups)
+        slices = h->window_h != kWindow ? 1 : pg.slices;
+        cta_cols = slices * (pg.cta_cols / pg.slices);
     } else {
         const int64_t need = (N + colw_ldg - 1) / colw_ldg;
         warps = need >= 8 ? 8 : need >= 4 ? 4 : need >= 2 ? (need > 2 ? 4 : 2) : 1;
@@ -1390,7 +1580,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
             DTC_CUDA(cudaMemsetAsync(h->counters, 0, ncnt * sizeof(int32_t), s));
             h->counters_len = ncnt;
         }
-        const size_t wsb = (size_t)h->num_slots * kWindow * npad * sizeof(float);
+        const size_t wsb = (size_t)h->num_slots * h->window_h * npad * sizeof(float);
         if (wsb > h->ws_bytes) {
             dfree(h->ws, s);
             h->ws_bytes = 0;

@@ -103,3 +103,26 @@ def test_invalid_inputs():
     with pytest.raises(DtcError) as e:
         build(2, 5, np.array([0, 3, 2], np.int32), np.array([0, 1, 2], np.int32), np.ones(3, np.float32))
     assert e.value.status == DTC_ERR_INVALID
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c3", "c4", "c5"])
+def test_tall_window_format_bit_exact(name):
+    """NEXT-2 layout (window_rows = 32): the GPU builder equals O2 applied to 32-row windows
+    (oracle.condense(window=32), pinned by the brute force and the decode round trip)."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=cfg.dtype, window_rows=32)
+    assert f.window_rows == 32
+    got = f.export()
+    assert_format_equal(got, oracle.condense(cfg.M, rp, ci, v, window=32))
+    check_units(got, cfg.M)
+
+
+def test_tall_window_fp16_unsupported():
+    from paper_conf_asplos_fan0024_b200 import DtcError, DTC_ERR_UNSUPPORTED
+    rp, ci = datagen.random_csr(40, 40, 0.1, 1)
+    v = datagen.uniform(1, 1, len(ci))
+    with pytest.raises(DtcError) as e:
+        build(40, 40, rp, ci, v, dtype="fp16", window_rows=32)
+    assert e.value.status == DTC_ERR_UNSUPPORTED

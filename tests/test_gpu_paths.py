@@ -23,6 +23,7 @@ VARIANTS = {
     "pers": {"kernel": "pad", "persistent": 1},
     "nofirst": {"kernel": "pad", "first_records": 0},
     "slice512": {"kernel": "pad", "slice_bytes": 512},
+    "tall": {},   # NEXT-2: 32-row windows (build option window_rows=32; TF32)
 }
 
 
@@ -32,6 +33,10 @@ def path(request):
 
 
 def build(*a, path=None, **kw):
+    if path == "tall":
+        if kw.get("dtype", "tf32") != "tf32":
+            pytest.skip("tall windows are TF32")
+        kw["window_rows"] = 32
     f = _build(*a, options=VARIANTS[path] if path else None, **kw)
     return f
 
@@ -51,6 +56,8 @@ def test_random_tolerance(path, dtype, N):
     # else the register gather
     elt = 2 if dtype == "fp16" else 4
     want = 1 if path == "ldg" or (N * elt) % 16 else 4
+    if path == "tall":
+        want = 4   # tall windows always run the padded kernel (B staged when TMA cannot describe it)
     assert f.get_option("last_kernel") == want
 
 

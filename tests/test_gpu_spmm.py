@@ -196,6 +196,20 @@ def test_config_full_size(name, N, parity_report):
     parity_report[f"{name} N={N} {cfg.dtype}"] = (worst, cfg.M * N)
 
 
+@pytest.mark.parametrize("name,N", [("c2", 128), ("c3", 256), ("c4", 128), ("c5", 512)])
+def test_tall_windows_full_size(name, N, parity_report):
+    """NEXT-2 layout (32-row windows, two 16-row tiles per TC block sharing the gathered B rows):
+    every element of C against O1 at full size."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = configs.make_B(cfg, N)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype=cfg.dtype, window_rows=32)
+    C = spmm(f, B)
+    worst = compare_chunked(C, cfg.M, cfg.K, rp, ci, v, B, cfg.dtype)
+    parity_report[f"{name} N={N} {cfg.dtype} tall32"] = (worst, cfg.M * N)
+
+
 @pytest.mark.parametrize("name,N", [("c3", 256), ("c3h", 256), ("c4", 128), ("c5", 512)])
 def test_p2_integer_full_size_exact(name, N, parity_report):
     """P2 at full size: integer A and B (|a|,|b| <= 2 -> every product and partial sum is exact in

@@ -63,25 +63,25 @@ def test_hand_worked_example():
     assert oracle.metcf_elements(20, 3, 20) == 36
 
 
-def brute_condense(M, K, rp, ci, vals):
-    """Dense-window brute force: scan k = 0..K-1, enumerate ids 0..127."""
+def brute_condense(M, K, rp, ci, vals, WH=16):
+    """Dense-window brute force: scan k = 0..K-1, enumerate ids 0..8*WH-1 (windows of WH rows)."""
     A = np.zeros((M, K), dtype=np.float64)
     mask = np.zeros((M, K), dtype=bool)
     for i in range(M):
         for p in range(rp[i], rp[i + 1]):
             A[i, ci[p]] = vals[p]
             mask[i, ci[p]] = True
-    W = -(-M // 16)
+    W = -(-M // WH)
     rwo, atob, tco, lid, tv = [0], [], [], [], []
     for w in range(W):
-        r0, r1 = 16 * w, min(16 * w + 16, M)
+        r0, r1 = WH * w, min(WH * w + WH, M)
         cols = [k for k in range(K) if mask[r0:r1, k].any()]
         nb = -(-len(cols) // 8)
         for b in range(nb):
             bc = cols[8 * b: 8 * b + 8]
             atob += bc + [-1] * (8 - len(bc))
             tco.append(len(lid))
-            for lid_ in range(128):
+            for lid_ in range(8 * WH):
                 r, c = divmod(lid_, 8)
                 if r0 + r < r1 and c < len(bc) and mask[r0 + r, bc[c]]:
                     lid.append(lid_)
@@ -95,11 +95,13 @@ def brute_condense(M, K, rp, ci, vals):
     (1, 1, 1.0, 1), (15, 9, 0.3, 2), (16, 8, 1.0, 3), (17, 40, 0.2, 4), (40, 70, 0.05, 5),
     (48, 130, 0.5, 6), (33, 300, 0.02, 7), (64, 12, 0.0, 8), (20, 200, 0.9, 9),
 ])
-def test_brute_force_condensation(M, K, density, seed):
+@pytest.mark.parametrize("WH", [16, 32])
+def test_brute_force_condensation(M, K, density, seed, WH):
+    """O2 (16-row ME-TCF and the 32-row windows of NEXT-2) against a dense brute force."""
     rp, ci = datagen.random_csr(M, K, density, seed)
     v = datagen.uniform(seed, 1, len(ci))
-    f = oracle.condense(M, rp, ci, v)
-    rwo, tco, lid, atob, tv = brute_condense(M, K, rp, ci, v)
+    f = oracle.condense(M, rp, ci, v, window=WH)
+    rwo, tco, lid, atob, tv = brute_condense(M, K, rp, ci, v, WH)
     assert f["row_window_offset"].tolist() == rwo
     assert f["tc_offset"].tolist() == tco
     assert f["tc_local_id"].tolist() == lid
@@ -107,14 +109,14 @@ def test_brute_force_condensation(M, K, density, seed):
     assert np.array_equal(f["tc_values"].astype(np.float64), np.array(tv, dtype=np.float64))
 
 
-def decode(M, f):
+def decode(M, f, WH=16):
     """ME-TCF -> (rows, cols, vals) sorted by (row, col)."""
     rwo, tco, lid = f["row_window_offset"], f["tc_offset"], f["tc_local_id"].astype(np.int64)
     atob, tv = f["sparse_a_to_b"], f["tc_values"]
     T = f["num_tc_blocks"]
     blk_of_window = np.repeat(np.arange(len(rwo) - 1), np.diff(rwo))
     blk_of_nnz = np.repeat(np.arange(T), np.diff(tco))
-    rows = 16 * blk_of_window[blk_of_nnz] + (lid >> 3)
+    rows = WH * blk_of_window[blk_of_nnz] + (lid >> 3)
     cols = atob[8 * blk_of_nnz + (lid & 7)]
     order = np.lexsort((cols, rows))
     return rows[order], cols[order], tv[order]
@@ -225,3 +227,15 @@ def test_p8_tcf_formula_reproduces_paper_percentage():
     # AvgRowL column = NNZ / M
     for m in t1.values():
         assert abs(m["nnz"] / m["M"] - m["avg_row_len"]) < 0.006
+
+
+@pytest.mark.parametrize("M,K,density,seed", [(100, 80, 0.05, 11), (77, 300, 0.3, 12), (64, 64, 1.0, 13)])
+def test_decode_round_trip_tall_windows(M, K, density, seed):
+    """32-row windows (NEXT-2): ids < 256 still fit uint8, and the decode reproduces the CSR."""
+    rp, ci = datagen.random_csr(M, K, density, seed)
+    v = datagen.uniform(seed, 1, len(ci))
+    f = oracle.condense(M, rp, ci, v, window=32)
+    rows, cols, vv = decode(M, f, WH=32)
+    ref_rows = np.repeat(np.arange(M), np.diff(rp))
+    assert np.array_equal(rows, ref_rows) and np.array_equal(cols, ci) and np.array_equal(vv, v)
+    assert f["num_windows"] == -(-M // 32) and int(f["tc_local_id"].max(initial=0)) < 256
