@@ -341,8 +341,8 @@ int dtc_partition_windows(const int32_t* rwo_host, int64_t num_windows, int32_t 
 /* Write a fresh 128-byte NCCL unique id to out128 (host). */
 int dtc_nccl_unique_id(void* out128);
 
-/* Collective over `world` ranks: condense the FULL csr (device pointers on this
- * rank's GPU) to find the window partition, then build this rank's local ME-TCF
+/* Collective over `world` ranks: count the FULL csr's TC blocks per window (F0-F2 only; device
+ * pointers on this rank's GPU) to find the window partition, then build this rank's local ME-TCF
  * from its CSR row slice.  nccl_id (host, 128 B, identical on all ranks) may be
  * NULL for a communicator-less local shard (single-GPU shard tests). */
 int dtc_dist_create(const dtc_csr_t* csr_full, int32_t rank, int32_t world, const void* nccl_id,
@@ -351,12 +351,24 @@ int dtc_dist_create(const dtc_csr_t* csr_full, int32_t rank, int32_t world, cons
 /* This rank's C rows [row_begin, row_end) and its local format handle (borrowed). */
 int dtc_dist_query(dtc_dist_t d, int64_t* row_begin, int64_t* row_end, dtc_handle_t* local);
 
-/* B: device K x N (ldb = N), valid on `root` (broadcast in place to the others).
- * C: device fp32; if gather_c, M x N (ldc = N) and every rank receives all rows;
- * else this rank's (row_end-row_begin) x N rows.  Needs a communicator unless
- * world == 1.  Stream-ordered.  Errors: INVALID, NCCL, CUDA. */
+/* B: device K x N (ldb = N), read on `root` only (other ranks may pass NULL; their B is not
+ * written).  The root packs B into column chunks (dtc_dist_chunks) of a library-owned buffer and
+ * broadcasts them with NCCL on a library stream while every rank's kernel computes the previous
+ * chunk's columns -- C(:, cols) depends only on B(:, cols), so C is bit-identical to one dtc_spmm
+ * over all N columns.  C: device fp32; if gather_c, M x N (ldc = N) and every rank receives all
+ * rows (grouped NCCL broadcasts per owner after the last chunk); else this rank's
+ * (row_end-row_begin) x N rows.  Without a communicator (nccl_id NULL) B must be resident and the
+ * call is a local dtc_spmm.  Stream-ordered on `stream`.  Errors: INVALID, NCCL, CUDA, OOM. */
 int dtc_spmm_dist(dtc_dist_t d, void* B, int32_t root, int64_t N, float* C, int32_t gather_c,
                   void* stream);
+
+/* HOST, pure: the column chunks of dtc_spmm_dist for K x N (elt bytes per element): widths are
+ * multiples of 32 columns, at most max_chunks (0 = 4, capped at 8), each >= 128 KB of B.
+ * col_begin int64[chunks+1].  Returns the number of chunks (>= 1) or INVALID. */
+int dtc_dist_chunks(int64_t K, int64_t N, int32_t elt, int32_t max_chunks, int64_t* col_begin);
+
+/* Override the chunk count of dtc_spmm_dist (0 = auto, 1 = unpipelined, up to 8).  Errors: INVALID. */
+int dtc_dist_set_chunks(dtc_dist_t d, int32_t chunks);
 
 void dtc_dist_destroy(dtc_dist_t d);
 

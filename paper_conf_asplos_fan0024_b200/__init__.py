@@ -14,7 +14,7 @@ from ._binding import (  # noqa: F401
     DTC_ERR_CUDA, DTC_ERR_NCCL, DTC_ERR_UNSUPPORTED, DTC_TF32, DTC_FP16,
     DtcError, Format, Dist, lib, library_path, exported_symbols, partition_windows, nccl_unique_id, tca_reorder,
     selector_ar, launches_per_call, version, OPTIONS, KERNELS, sched_model, make_model, selector_plan,
-    selector_simulate, selector_report, SchedModel, softmax_xent, sgd_update, GCN2, tca_reorder_checked,
+    selector_simulate, selector_report, SchedModel, softmax_xent, sgd_update, GCN2, tca_reorder_checked, dist_chunks,
 )
 
 __all__ = ["Format", "Dist", "DtcError", "lib", "partition_windows", "nccl_unique_id"]

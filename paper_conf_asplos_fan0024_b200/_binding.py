@@ -115,6 +115,8 @@ def lib():
             L.dtc_dist_create.argtypes = [P(_Csr), _i32, _i32, _vp, _vp, P(_vp)]
             L.dtc_dist_query.argtypes = [_vp, P(_i64), P(_i64), P(_vp)]
             L.dtc_spmm_dist.argtypes = [_vp, _vp, _i32, _i64, _vp, _i32, _vp]
+            L.dtc_dist_chunks.argtypes = [_i64, _i64, _i32, _i32, _vp]
+            L.dtc_dist_set_chunks.argtypes = [_vp, _i32]
             L.dtc_dist_destroy.argtypes = [_vp]
             L.dtc_dist_destroy.restype = None
             L.dtc_status_string.argtypes = [ctypes.c_int]
@@ -565,6 +567,15 @@ def tca_reorder_checked(M: int, K: int, rowptr, colidx, sm_num: int = 148):
     return perm[:M], {"T_identity": t0.value, "T_reordered": t1.value, "applied": bool(ap.value)}
 
 
+def dist_chunks(K: int, N: int, elt: int, max_chunks: int = 0) -> np.ndarray:
+    """Column chunk boundaries of dtc_spmm_dist's pipelined broadcast (dtc_dist_chunks, host)."""
+    out = np.zeros(9, dtype=np.int64)
+    n = lib().dtc_dist_chunks(int(K), int(N), int(elt), int(max_chunks), out.ctypes.data_as(_vp))
+    if n < 1:
+        _check(n, "dtc_dist_chunks")
+    return out[: n + 1]
+
+
 def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().dtc_nccl_unique_id(buf), "dtc_nccl_unique_id")
@@ -603,11 +614,19 @@ class Dist:
         _check(lib().dtc_spmm(self._local, _dptr(B), N, N, _dptr(C_local), N, _stream_ptr(stream)), "dtc_spmm")
         return C_local
 
-    def spmm(self, B, C, root: int = 0, gather_c: bool = True, stream=None):
-        """dtc_spmm_dist: B (K x N, valid on root) is broadcast; C is M x N (gather_c) or this rank's rows."""
+    def set_chunks(self, chunks: int) -> None:
+        """Column chunks of the pipelined broadcast (dtc_dist_set_chunks): 0 = auto, 1 = unpipelined."""
+        _check(lib().dtc_dist_set_chunks(self._h, int(chunks)), "dtc_dist_set_chunks")
+
+    def spmm(self, B, C, root: int = 0, gather_c: bool = True, stream=None, N: int | None = None):
+        """dtc_spmm_dist: B (K x N) is read on root only (None elsewhere, then pass N) and broadcast in
+        column chunks pipelined with the kernel; C is M x N (gather_c) or this rank's rows."""
         import torch
-        _dense(B, "B", (self.K, None), self._want())
-        N = B.shape[1]
+        if B is not None:
+            _dense(B, "B", (self.K, None), self._want())
+            N = B.shape[1]
+        elif N is None or self.rank == root:
+            raise ValueError("B is required on the root (elsewhere pass N)")
         rows = self.M if gather_c else max(self.row_end - self.row_begin, 1)
         _dense(C, "C", (rows, N), torch.float32)
         _check(lib().dtc_spmm_dist(self._h, _dptr(B), root, N, _dptr(C), int(gather_c), _stream_ptr(stream)),

@@ -847,6 +847,66 @@ fail:
 #undef TRYC
 }
 
+// F0-F2 only: validate the CSR and count each 16-row window's TC blocks, returning RowWindowOffset on
+// the host -- all the multi-GPU partitioner needs (no SparseAtoB / values / units are built).
+int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out) {
+    if (!csr || !rwo_out) { set_error("null argument"); return DTC_ERR_INVALID; }
+    const int64_t M = csr->M, K = csr->K, nnz = csr->nnz;
+    if (M < 0 || K < 0 || nnz < 0 || nnz >= INT32_MAX || M >= INT32_MAX - 16 || K >= INT32_MAX || !csr->rowptr ||
+        (nnz > 0 && !csr->colidx)) {
+        set_error("bad CSR");
+        return DTC_ERR_INVALID;
+    }
+    const int64_t W = (M + kWindow - 1) / kWindow;
+    int* flags = nullptr;
+    int32_t *u = nullptr, *uniq = nullptr, *rank = nullptr;
+    int64_t *nb = nullptr, *tmp = nullptr;
+    int rc = DTC_OK;
+    std::vector<int64_t> h((size_t)W + 1, 0);
+    int hflags = 0;
+#define TRY(x) do { rc = (x); if (rc != DTC_OK) goto done; } while (0)
+#define TRYC(x) do { cudaError_t _e = (x); if (_e != cudaSuccess) { rc = cuda_fail(_e, #x, __FILE__, __LINE__); goto done; } } while (0)
+    TRY(dalloc(&flags, 1, s));
+    TRYC(cudaMemsetAsync(flags, 0, sizeof(int), s));
+    TRY(dalloc(&u, W + 1, s));
+    TRY(dalloc(&nb, W + 1, s));
+    TRY(dalloc(&uniq, nnz, s));
+    TRY(dalloc(&rank, nnz, s));
+    TRY(dalloc(&tmp, scan_tmp_elems(W + 1) + 64, s));
+    if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, flags);
+    if (W > 0) {
+        const size_t bm_smem = 2 * kBmWords * sizeof(uint32_t);
+        k_dedup_sort<16><<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq, rank);
+        TRYC(cudaFuncSetAttribute(k_dedup_bitmap<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+        k_dedup_bitmap<16><<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq,
+                                                                   rank);
+        exclusive_scan_i64(nb, nb, W, tmp, s);
+    } else {
+        TRYC(cudaMemsetAsync(nb, 0, sizeof(int64_t), s));
+    }
+    TRYC(cudaGetLastError());
+    TRYC(cudaMemcpyAsync(h.data(), nb, (W + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    TRYC(cudaMemcpyAsync(&hflags, flags, sizeof(int), cudaMemcpyDeviceToHost, s));
+    TRYC(cudaStreamSynchronize(s));
+    if (hflags) {
+        if (hflags & F_INVALID) { set_error("malformed rowptr"); rc = DTC_ERR_INVALID; }
+        else if (hflags & F_RANGE) { set_error("column index out of [0, K)"); rc = DTC_ERR_RANGE; }
+        else if (hflags & F_DUPLICATE) { set_error("duplicate column within a row"); rc = DTC_ERR_DUPLICATE; }
+        else { set_error("columns not ascending within a row"); rc = DTC_ERR_UNSORTED; }
+        goto done;
+    }
+    if (h[W] >= INT32_MAX / 8) { set_error("NumTCBlock too large"); rc = DTC_ERR_UNSUPPORTED; goto done; }
+    rwo_out->assign((size_t)W + 1, 0);
+    for (int64_t w = 0; w <= W; ++w) (*rwo_out)[(size_t)w] = (int32_t)h[(size_t)w];
+done:
+    cudaGetLastError();
+    dfree(flags, s); dfree(u, s); dfree(nb, s); dfree(uniq, s); dfree(rank, s); dfree(tmp, s);
+    cudaStreamSynchronize(s);
+    return rc;
+#undef TRY
+#undef TRYC
+}
+
 }  // namespace dtc
 
 using namespace dtc;

@@ -5,6 +5,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <string>
+#include <vector>
 
 #include "../../include/dtc.h"
 
@@ -153,6 +154,9 @@ int pad_occupancy(int dtype, int64_t N, int window_h = 16);
 int selector_plan(const int32_t* rwo, int64_t W, const dtc_sched_model_t& m, const int32_t* cand, int ncand,
                   int guided_opt, dtc_plan_t* plans, dtc_plan_t* best);
 int sched_model(int dtype, int64_t N, dtc_sched_model_t* m, int window_h = 16);
+
+// F0-F2 only (dtc_format.cu): validated RowWindowOffset of 16-row windows, on the host
+int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out);
 
 // internal build used by the distributed layer: optional row range of the csr
 int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s,
