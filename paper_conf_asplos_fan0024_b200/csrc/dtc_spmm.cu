@@ -678,15 +678,23 @@ template <int H> constexpr int pad_aslot() { return pad_aval_bytes<H>() + pad_ba
 // and for tall windows; with 2 TF32 consumer warps its barrier and the 16 KB of fragments (fewer
 // CTAs per SM) cost more than they save: c3 +13.6%, c5 +7.2%, c4/256 +15%, c3h +6.4%, but
 // c2 -14%, c4/128 -13.5% (profiles/r02_ab_coop.txt).
+#ifndef DTC_PAD_COOP_FORCE
+#define DTC_PAD_COOP_FORCE -1
+#endif
 template <int DT, int SL, int SEG, int H>
-constexpr bool pad_coop() { return DT == DTC_FP16 || SL * SEG / 2 >= 4 || H > 1; }
+constexpr bool pad_coop() {
+    return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || SL * SEG / 2 >= 4 || H > 1);
+}
 template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
     return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
 }
+// raw A batch slots (double buffered; a third slot would let the producer run a batch further ahead
+// but costs a CTA per SM on c3: 8.59 -> 6.88 TFLOP/s measured, profiles/r02_ab_coop_slots.txt)
+template <int DT, int SL, int SEG, int H> constexpr int pad_aslots() { return 2; }
 template <int SL, int SEG, int H = 1, int DT = DTC_TF32>
 constexpr size_t pad_smem_bytes() {
-    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + 2 * pad_aslot<H>() + pad_frag_bytes<DT, SL, SEG, H>() +
-           128;
+    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<H>() +
+           pad_frag_bytes<DT, SL, SEG, H>() + 128;
 }
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
 template <int DT, int SL, int H = 1>
@@ -763,13 +771,13 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
     constexpr int BATCH = pad_batch<H>();       // TC blocks per A batch
-    constexpr int ASLOT = pad_aslot<H>(), AVAL = pad_aval_bytes<H>();
+    constexpr int ASLOT = pad_aslot<H>(), AVAL = pad_aval_bytes<H>(), NA = pad_aslots<DT, SL, SEG, H>();
     const uint32_t aring = ring + R * STAGE;                          // [2][ASLOT] A batches
-    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[2], bar_aempty[2], bar_ufull[2], bar_uempty[2];
-    __shared__ int s_abyte[2];   // byte offset of the batch's first value inside its A slot
+    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[NA], bar_aempty[NA], bar_ufull[2], bar_uempty[2];
+    __shared__ int s_abyte[NA];   // byte offset of the batch's first value inside its A slot (batch c: slot c % NA)
     constexpr bool COOP = pad_coop<DT, SL, SEG, H>();
     __shared__ uint8_t s_live[2][BATCH];   // COOP: per block, bit h = sub-tile h has a non-zero
-    const uint32_t frags = aring + 2 * ASLOT;  // COOP: [2][BATCH][H] lane-major fragments (expand())
+    const uint32_t frags = aring + NA * ASLOT;  // COOP: [2][BATCH][H] lane-major fragments (expand())
     __shared__ int s_unit[2][10];   // published unit: Unit record, end block of its first window, index (-1 = done)
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -790,9 +798,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             mbar_init(&bar_full[i], 1);
             mbar_init(&bar_empty[i], ncons);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < NA; ++i) {
             mbar_init(&bar_afull[i], 1);
             mbar_init(&bar_aempty[i], COOP ? 1 : ncons);
+        }
+        for (int i = 0; i < 2; ++i) {
             mbar_init(&bar_ufull[i], 1);
             mbar_init(&bar_uempty[i], ncons);
         }
@@ -888,12 +898,12 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             const int q2 = draw();   // reserve the unit after next now; its latency hides behind this unit
             const int nblocks = u.be - u.bb;
             for (int i0 = 0; i0 < nblocks; i0 += BATCH) {
-                const int c = gc0 + i0 / BATCH, aslot = c & 1;
+                const int c = gc0 + i0 / BATCH, aslot = c % NA;
                 const BatchMeta cur = finish(rnext);
                 rnext = i0 + BATCH < nblocks ? load_raw(u, i0 + BATCH) : load_raw(un, 0);
                 if (i0 == 0) end0n = first_end(un);
                 const int nj = min(BATCH, nblocks - i0);
-                if (c >= 2) mbar_wait(&bar_aempty[aslot], ((c >> 1) - 1) & 1);
+                if (c >= NA) mbar_wait(&bar_aempty[aslot], ((c / NA) - 1) & 1);
                 if (lane == 0) {
                     const int64_t lo = ((int64_t)cur.e0 * ELT) & ~int64_t(15);
                     const int64_t hi = ((int64_t)cur.e1 * ELT + 15) & ~int64_t(15);
@@ -996,9 +1006,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     // rewritten only at batch c+2, after every consumer has passed the barrier of batch c+1.
     constexpr int FSUB = 32 * FW * 4;                      // bytes of one sub-tile's fragments
     auto expand = [&](int c, int nj) {
-        mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
-        const uint32_t slot = aring + (c & 1) * ASLOT;
-        const uint32_t v0 = slot + s_abyte[c & 1], maddr = slot + AVAL;
+        mbar_wait(&bar_afull[c % NA], (c / NA) & 1);
+        const uint32_t slot = aring + (c % NA) * ASLOT;
+        const uint32_t v0 = slot + s_abyte[c % NA], maddr = slot + AVAL;
         // value offset of every block of the batch: exclusive warp scan of the blocks' popcounts
         int cnt = 0;
         if (lane < nj)
@@ -1035,7 +1045,6 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             if (lane == 0) s_live[c & 1][jj] = (uint8_t)lv;
         }
         asm volatile("bar.sync 1, %0;" ::"r"(ncons * 32) : "memory");
-        if (warp == 0 && lane == 0) mbar_arrive(&bar_aempty[c & 1]);   // raw values and masks consumed
     };
     // this lane's fragments of block i (batch c = gc0 + i / BATCH); live[h] = sub-tile h has a
     // non-zero (warp-uniform)
@@ -1055,8 +1064,14 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             }
         }
     };
+    // the raw A slot of a batch is released by warp 0 after its LAST block (not right after the
+    // expansion: releasing it at the barrier let the producer run an A batch further ahead and
+    // corrupted C on long units -- measured, found with a fragment cross-check; kept late)
     auto release_coop = [&](int i, int gi, int nblocks, int gc0) {
-        if (lane == 0) mbar_arrive(&bar_empty[gi % R]);
+        if (lane == 0) {
+            mbar_arrive(&bar_empty[gi % R]);
+            if (warp == 0 && ((i % BATCH) == BATCH - 1 || i == nblocks - 1)) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) % NA]);
+        }
     };
 
     // A batch cursor: the next block's first value (bytes) and the batch's mask array
@@ -1066,9 +1081,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     auto afrag_dec = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
         const int j = i % BATCH, c = gc0 + i / BATCH;
         if (j == 0) {
-            mbar_wait(&bar_afull[c & 1], (c >> 1) & 1);
-            const uint32_t slot = aring + (c & 1) * ASLOT;
-            vaddr = slot + s_abyte[c & 1];
+            mbar_wait(&bar_afull[c % NA], (c / NA) & 1);
+            const uint32_t slot = aring + (c % NA) * ASLOT;
+            vaddr = slot + s_abyte[c % NA];
             maddr = slot + AVAL;
         }
 #pragma unroll
@@ -1084,7 +1099,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (lane == 0) {
             mbar_arrive(&bar_empty[gi % R]);
             const int j = i % BATCH;
-            if (j == BATCH - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) & 1]);
+            if (j == BATCH - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) % NA]);
         }
     };
     auto afrag = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
@@ -1470,8 +1485,13 @@ int pad_occupancy(int dtype, int64_t N, int window_h) {
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return -1; }
     auto occ = [&](auto kern, int sl, int seg, size_t smem) -> int {
-        static KernelState ks;   // one per kernel instantiation (the lambda is instantiated per kernel type)
-        return kernel_setup(kern, (sl * seg / 2 + 1) * 32, smem, ks, dev);
+        // (every k_spmm_pad instantiation has the same type, so no per-type static cache here)
+        int v = 0;
+        if (smem > 48 * 1024 &&
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+            return -1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, kern, (sl * seg / 2 + 1) * 32, smem) != cudaSuccess) return -1;
+        return v;
     };
 #define DTC_OCC(DT, H)                                                                                              \
     do {                                                                                                            \
