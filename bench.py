@@ -68,8 +68,9 @@ def parse_args():
     p.add_argument("--persistent", type=int, default=0, help="DTC_OPT_PERSISTENT for the timed launches")
     p.add_argument("--window-rows", type=int, default=0,
                    help="32: NEXT-2 tall windows (TF32 workloads; FP16 legs keep 16-row ME-TCF)")
-    p.add_argument("--selector", type=int, default=0,
-                   help="F4 cut by the B200 Selector's plan for this N (NEXT-4, dtc_selector_plan): 1 on, 0 fixed rule")
+    p.add_argument("--selector", type=int, default=2,
+                   help="B200 Selector (NEXT-4): 1 = plan U by simulation + window height, 2 = window height only "
+                        "(32-row NEXT-2 windows where they pay), 0 = fixed rule, 16-row windows")
     p.add_argument("--ncu", default="auto", choices=["auto", "off"],
                    help="capture DRAM traffic of one launch per leg under ncu (subprocess)")
     p.add_argument("--no-cusparse", action="store_true")
@@ -375,7 +376,8 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
     leg.update({"num_tc_blocks": T, "mean_nnz_tc": round(nnz / max(T, 1), 3), "sum_u": ab["sum_u"],
                 "unit_blocks": fmt.unit_blocks, "num_units": fmt.num_units,
                 "split_windows": fmt.num_split_windows, "guided": fmt.get_option("guided"),
-                "f4_plan": "selector" if args.selector else "rule", "window_rows": fmt.window_rows,
+                "f4_plan": {0: "rule", 1: "selector", 2: "rule + selector window height"}[args.selector],
+                "window_rows": fmt.window_rows,
                 "selector_predicted_ms": round(fmt.get_option("plan_makespan_ns") / 1e6, 4) or None,
                 "format_build_ms": round(build_ms_runs[-1], 3),
                 "format_build_first_call_ms": round(build_ms_runs[0], 3),

@@ -103,6 +103,11 @@ typedef struct {
     /* B200 Selector (NEXT-4, dtc_selector_plan): with unit_blocks = 0 and selector = 1, F4 takes the
      * unit size and guided tail whose simulated launch for N = n_hint columns (0 = 128) is shortest;
      * selector = 0 keeps the fixed rule (U = clamp(2T/W, 64, 256), at most T/(24 SMs); guided as above).
+     * With selector = 1 or 2, window_rows = 0 and a TF32 matrix whose gathered rows are >= 1 KB
+     * (n_hint x 4 >= 1024), it also picks the window height: 32 rows (NEXT-2) when that lowers the TC
+     * blocks to <= 0.65 of the 16-row count (F0-F2 run at both heights first); selector = 2 picks
+     * only the window height and keeps the fixed unit-size rule (the simulated U plan ignores L2
+     * locality and lost 4% on the products-shaped c5).
      * Same C either way (within tolerance; integer inputs bit-exact). */
     int32_t n_hint;
     int32_t selector;

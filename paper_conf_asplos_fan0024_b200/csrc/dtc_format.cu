@@ -582,8 +582,21 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
     if (transpose && opts->row_perm) { set_error("transpose and row_perm cannot be combined"); return DTC_ERR_INVALID; }
     // the condensed matrix: A (M x K) or A^T (K x M)
     const int64_t Mc = transpose ? K : M, Kc = transpose ? M : K;
-    const int WH = (opts && opts->window_rows > 0) ? opts->window_rows : kWindow;
+    int WH = (opts && opts->window_rows > 0) ? opts->window_rows : kWindow;
     if (WH != 16 && WH != 32) { set_error("window_rows must be 16 or 32"); return DTC_ERR_INVALID; }
+    // Selector, window height (NEXT-2): 32-row windows pay when two 16-row windows share >= 35% of
+    // their gathered B rows (T32 <= 0.65 T16) and each gathered row is >= 1 KB, so the saved bytes
+    // outweigh the doubled MMA / fragment work (c4 N=256: +17%; every other workload loses;
+    // profiles/r02_ab_tall_windows.txt).  TF32 only; needs F0-F2 at both heights (two extra passes).
+    if (opts && opts->selector > 0 && opts->window_rows == 0 && csr->dtype == DTC_TF32 && !transpose &&
+        !opts->row_perm && (int64_t)(opts->n_hint > 0 ? opts->n_hint : 128) * 4 >= 1024 && csr->nnz > 0) {
+        std::vector<int32_t> r16, r32;
+        int rc0 = window_offsets(csr, s, &r16, 16);
+        if (rc0 == DTC_OK) rc0 = window_offsets(csr, s, &r32, 32);
+        if (rc0 != DTC_OK) return rc0;
+        const double t16 = (double)r16.back(), t32 = (double)r32.back();
+        if (t16 > 0 && t32 <= 0.65 * t16) WH = 32;
+    }
     if (WH == 32 && csr->dtype != DTC_TF32) { set_error("window_rows = 32 is implemented for TF32"); return DTC_ERR_UNSUPPORTED; }
     const int64_t W = (Mc + WH - 1) / WH;
 
@@ -776,7 +789,7 @@ int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_
         // B200 Selector (NEXT-4, dtc_selector.cu): with no unit size given, simulate the launch of
         // every candidate plan (U x guided tail) for the expected N and keep the shortest
         const int sel = opts ? opts->selector : 0;
-        if (!(opts && opts->unit_blocks > 0) && sel > 0 && T > 0) {
+        if (!(opts && opts->unit_blocks > 0) && sel == 1 && T > 0) {
             std::vector<int32_t> hrwo((size_t)W + 1);
             TRYC(cudaMemcpyAsync(hrwo.data(), h->rwo, (W + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
             TRYC(cudaStreamSynchronize(s));
@@ -849,7 +862,7 @@ fail:
 
 // F0-F2 only: validate the CSR and count each 16-row window's TC blocks, returning RowWindowOffset on
 // the host -- all the multi-GPU partitioner needs (no SparseAtoB / values / units are built).
-int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out) {
+int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out, int WH) {
     if (!csr || !rwo_out) { set_error("null argument"); return DTC_ERR_INVALID; }
     const int64_t M = csr->M, K = csr->K, nnz = csr->nnz;
     if (M < 0 || K < 0 || nnz < 0 || nnz >= INT32_MAX || M >= INT32_MAX - 16 || K >= INT32_MAX || !csr->rowptr ||
@@ -857,7 +870,8 @@ int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* r
         set_error("bad CSR");
         return DTC_ERR_INVALID;
     }
-    const int64_t W = (M + kWindow - 1) / kWindow;
+    if (WH != 16 && WH != 32) { set_error("window height %d", WH); return DTC_ERR_INVALID; }
+    const int64_t W = (M + WH - 1) / WH;
     int* flags = nullptr;
     int32_t *u = nullptr, *uniq = nullptr, *rank = nullptr;
     int64_t *nb = nullptr, *tmp = nullptr;
@@ -876,10 +890,17 @@ int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* r
     if (M > 0) k_validate<<<grid_for(M * 32, 256, 148 * 64), 256, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, flags);
     if (W > 0) {
         const size_t bm_smem = 2 * kBmWords * sizeof(uint32_t);
-        k_dedup_sort<16><<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq, rank);
-        TRYC(cudaFuncSetAttribute(k_dedup_bitmap<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
-        k_dedup_bitmap<16><<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq,
-                                                                   rank);
+        if (WH == 16) {
+            k_dedup_sort<16><<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq, rank);
+            TRYC(cudaFuncSetAttribute(k_dedup_bitmap<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+            k_dedup_bitmap<16><<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb,
+                                                                       uniq, rank);
+        } else {
+            k_dedup_sort<32><<<(unsigned)W, kSortThreads, 0, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb, uniq, rank);
+            TRYC(cudaFuncSetAttribute(k_dedup_bitmap<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem));
+            k_dedup_bitmap<32><<<(unsigned)W, kBmThreads, bm_smem, s>>>(M, K, nnz, csr->rowptr, csr->colidx, 0, u, nb,
+                                                                       uniq, rank);
+        }
         exclusive_scan_i64(nb, nb, W, tmp, s);
     } else {
         TRYC(cudaMemsetAsync(nb, 0, sizeof(int64_t), s));

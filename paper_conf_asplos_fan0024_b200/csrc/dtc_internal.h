@@ -156,7 +156,7 @@ int selector_plan(const int32_t* rwo, int64_t W, const dtc_sched_model_t& m, con
 int sched_model(int dtype, int64_t N, dtc_sched_model_t* m, int window_h = 16);
 
 // F0-F2 only (dtc_format.cu): validated RowWindowOffset of 16-row windows, on the host
-int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out);
+int window_offsets(const dtc_csr_t* csr, cudaStream_t s, std::vector<int32_t>* rwo_out, int window_h = 16);
 
 // internal build used by the distributed layer: optional row range of the csr
 int format_build(const dtc_csr_t* csr, const dtc_build_opts_t* opts, cudaStream_t s,

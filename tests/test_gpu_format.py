@@ -126,3 +126,18 @@ def test_tall_window_fp16_unsupported():
     with pytest.raises(DtcError) as e:
         build(40, 40, rp, ci, v, dtype="fp16", window_rows=32)
     assert e.value.status == DTC_ERR_UNSUPPORTED
+
+
+@pytest.mark.parametrize("name,N,want", [("c4", 256, 32), ("c4", 128, 16), ("c2", 256, 16), ("c1", 512, 16)])
+def test_selector_picks_window_height(name, N, want):
+    """Selector (selector=1, window_rows=0): 32-row windows exactly when T32 <= 0.65 T16 and the
+    gathered rows are >= 1 KB (n_hint x 4 B); the counts come from O2 at both heights."""
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    f = build(cfg.M, cfg.K, rp, ci, v, selector=2, n_hint=N)
+    _, t16 = oracle.condense_count(cfg.M, rp, ci, 16)
+    _, t32 = oracle.condense_count(cfg.M, rp, ci, 32)
+    expect = 32 if (N * 4 >= 1024 and t32 <= 0.65 * t16) else 16
+    assert f.window_rows == expect == want
+    assert_format_equal(f.export(), oracle.condense(cfg.M, rp, ci, v, window=expect))
