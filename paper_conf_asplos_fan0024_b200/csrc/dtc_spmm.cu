@@ -670,9 +670,12 @@ static_assert((kFirstRec * 4) % 16 == 0, "int4 loads of the side record");
 // A batch slot for windows of H x 16 rows: values (<= batch x 128H x 4 B + 16, 128-aligned), then
 // one 16H-byte occupancy mask per block
 // (tall windows take batches of kPadBatch / H blocks, so a batch slot is the same size for every H)
-template <int H> constexpr int pad_batch() { return kPadBatch / H; }
-template <int H> constexpr int pad_aval_bytes() { return pad_batch<H>() * 512 * H + 128; }
-template <int H> constexpr int pad_aslot() { return pad_aval_bytes<H>() + pad_batch<H>() * 16 * H; }
+#ifndef DTC_PAD_TF32_BATCH
+#define DTC_PAD_TF32_BATCH 16
+#endif
+template <int DT, int H> constexpr int pad_batch() { return (DT == DTC_TF32 ? DTC_PAD_TF32_BATCH : kPadBatch) / H; }
+template <int DT, int H> constexpr int pad_aval_bytes() { return pad_batch<DT, H>() * 512 * H + 128; }
+template <int DT, int H> constexpr int pad_aslot() { return pad_aval_bytes<DT, H>() + pad_batch<DT, H>() * 16 * H; }
 // Cooperative A expansion (consumers decode each block once into shared memory) pays where a
 // CTA has >= 4 consumer warps (each would otherwise decode every block), for FP16 (block pairs),
 // and for tall windows; with 2 TF32 consumer warps its barrier and the 16 KB of fragments (fewer
@@ -686,14 +689,14 @@ constexpr bool pad_coop() {
     return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || SL * SEG / 2 >= 4 || H > 1);
 }
 template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
-    return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
+    return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<DT, H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
 }
 // raw A batch slots (double buffered; a third slot would let the producer run a batch further ahead
 // but costs a CTA per SM on c3: 8.59 -> 6.88 TFLOP/s measured, profiles/r02_ab_coop_slots.txt)
 template <int DT, int SL, int SEG, int H> constexpr int pad_aslots() { return 2; }
 template <int SL, int SEG, int H = 1, int DT = DTC_TF32>
 constexpr size_t pad_smem_bytes() {
-    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<H>() +
+    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<DT, H>() +
            pad_frag_bytes<DT, SL, SEG, H>() + 128;
 }
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
@@ -740,7 +743,7 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
     return (uint32_t)v;
 }
 
-template <int DT, int SL, int SEG, bool VEC, int H>
+template <int DT, int SL, int SEG, bool VEC, int H, bool TRACE = false>
 // (min-blocks form of the register cap: measured 8-13% faster than __maxnreg__ with the same cap,
 // profiles/r02_ab_launch_bounds.txt)
 __global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL, H>()))
@@ -770,8 +773,8 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     constexpr int SLICE_COLS = SEG * COLW1;    // 128 / 256 fp32 or 256 / 512 fp16 columns per slice
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
-    constexpr int BATCH = pad_batch<H>();       // TC blocks per A batch
-    constexpr int ASLOT = pad_aslot<H>(), AVAL = pad_aval_bytes<H>(), NA = pad_aslots<DT, SL, SEG, H>();
+    constexpr int BATCH = pad_batch<DT, H>();   // TC blocks per A batch
+    constexpr int ASLOT = pad_aslot<DT, H>(), AVAL = pad_aval_bytes<DT, H>(), NA = pad_aslots<DT, SL, SEG, H>();
     const uint32_t aring = ring + R * STAGE;                          // [2][ASLOT] A batches
     __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[NA], bar_aempty[NA], bar_ufull[2], bar_uempty[2];
     __shared__ int s_abyte[NA];   // byte offset of the batch's first value inside its A slot (batch c: slot c % NA)
@@ -921,7 +924,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                 for (int j = 0; j < nj; ++j) {
                     const int i = gi0 + i0 + j, s = i % R;
                     if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
-                    if (tr && i == 0 && lane == 0) tr[3] = gtimer();
+                    if (TRACE && tr && i == 0 && lane == 0) tr[3] = gtimer();
                     if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
                     __syncwarp();
                     if (jl == j) {
@@ -1165,7 +1168,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             if (pair) afrag(i + 1, gc0, a2, live2);
             // S2/S3: B fragments from the padded stage(s), mma (a sub-tile without non-zeros is skipped)
             mbar_wait(&bar_full[s], (gi / R) & 1);
-            if (tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();
+            if (TRACE && tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();   // (compiled out unless traced)
             const uint32_t st = ring + s * STAGE;
             if constexpr (DT == DTC_TF32) {
 #pragma unroll
@@ -1379,7 +1382,8 @@ static cudaError_t first_records(dtc_format* h, cudaStream_t s) {
     int32_t* d = nullptr;
     if (dalloc(&d, (size_t)h->num_units * kFirstRec, s) != DTC_OK) return cudaErrorMemoryAllocation;
     k_units_first<<<(unsigned)std::min<int64_t>(h->num_units, 65535), 128, 0, s>>>(
-        h->num_units, h->units, h->atob, h->tco, h->rwo, d, h->window_h == kWindow ? pad_batch<1>() : pad_batch<2>());
+        h->num_units, h->units, h->atob, h->tco, h->rwo, d,
+        h->dtype == DTC_FP16 ? pad_batch<DTC_FP16, 1>() : (h->window_h == kWindow ? pad_batch<DTC_TF32, 1>() : pad_batch<DTC_TF32, 2>()));
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { dfree(d, s); return e; }
     h->ufirst = d;
@@ -1445,6 +1449,15 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     }
     const dim3 grid((unsigned)gx, (unsigned)a.gy);
     int64_t* trace = (h->trace && (int64_t)grid.x * grid.y <= h->trace_cap) ? h->trace : nullptr;
+    if (trace) {   // traced launch: the instantiation that records the per-block timestamps too
+        static KernelState kst;
+        if (kernel_setup(k_spmm_pad<DT, SL, SEG, VEC, H, true>, threads, smem, kst, a.h->device) < 0)
+            return cudaErrorInvalidConfiguration;
+        k_spmm_pad<DT, SL, SEG, VEC, H, true><<<grid, threads, smem, a.s>>>(
+            map, units, h->rwo, h->tco, reinterpret_cast<const uint4*>(h->mask), h->atob, h->vals, a.C, a.ldc, h->M, a.N,
+            h->ws, h->counters, a.npad, h->rowmap, trace, (int)h->num_units, uctr, a.te, ufirst);
+        return cudaGetLastError();
+    }
     k_spmm_pad<DT, SL, SEG, VEC, H><<<grid, threads, smem, a.s>>>(
         map, units, h->rwo, h->tco, reinterpret_cast<const uint4*>(h->mask), h->atob, h->vals, a.C, a.ldc, h->M, a.N,
         h->ws, h->counters, a.npad, h->rowmap, trace, (int)h->num_units, uctr, a.te, ufirst);

@@ -18,6 +18,7 @@ for c in c3 c2 c3h c4 c5; do
   python tools/ncu_summary.py /tmp/ncu/ev_prof_$c.ncu-rep > gpurun_out/ev_ncu_$c.txt 2>&1
   ncu -i /tmp/ncu/ev_prof_$c.ncu-rep --page raw --csv > gpurun_out/ev_raw_$c.csv 2>/dev/null
   timeout 300 python tools/trace_cta.py $c > gpurun_out/ev_trace_$c.txt 2>&1
+  timeout 300 python tools/trace_cta.py $c --persistent 1 > gpurun_out/ev_trace_pers_$c.txt 2>&1
 done
 ncu -i /tmp/ncu/ev_prof_c3.ncu-rep --page source --csv > gpurun_out/ev_source_c3.csv 2>/dev/null
 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/ev_smoke.txt 2>&1
