@@ -758,7 +758,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     constexpr int ELT = (int)sizeof(typename Tr::elt);
     // optional per-CTA timeline (dtc_format_set_trace): {cta, smid, t_start, t_first_issue,
     // t_first_data, t_consumer_done, nblocks, t_producer_done} in %globaltimer ns
-    int64_t* tr = trace ? trace + ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * 8 : nullptr;
+    int64_t* tr = (TRACE && trace) ? trace + ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * 8 : nullptr;   // TRACE instantiation only
     if (tr && threadIdx.x == 0) {
         tr[0] = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
         tr[1] = smid();
