@@ -141,3 +141,22 @@ def test_selector_picks_window_height(name, N, want):
     expect = 32 if (N * 4 >= 1024 and t32 <= 0.65 * t16) else 16
     assert f.window_rows == expect == want
     assert_format_equal(f.export(), oracle.condense(cfg.M, rp, ci, v, window=expect))
+
+
+@pytest.mark.parametrize("U", [16, 64, 256])
+@pytest.mark.parametrize("guided", [1, -1])
+@pytest.mark.parametrize("name", ["c2", "c4"])
+def test_selector_plans_the_builders_units(name, U, guided):
+    """The Selector simulates exactly the units F4 emits: its unit count for (U, guided) equals the
+    builder's, and its simulated makespan equals dtc_selector_simulate over the exported units."""
+    import paper_conf_asplos_fan0024_b200 as dtc
+    cfg = configs.get(name)
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    f = build(cfg.M, cfg.K, rp, ci, v, unit_blocks=U, guided=guided)
+    e = f.export()
+    m = dtc.sched_model("tf32", cfg.N)
+    plan = dtc.selector_plan(e["row_window_offset"], m, [U], guided=guided)
+    p = [x for x in plan["plans"] if x["makespan_ns"] >= 0][0]
+    assert p["num_units"] == f.num_units
+    assert p["makespan_ns"] == pytest.approx(dtc.selector_simulate(e["units"], m), rel=1e-12)

@@ -86,3 +86,51 @@ def test_native_rejects_bad_arguments():
             dtc.selector_ar(rwo, S, O)
     with pytest.raises(dtc.DtcError):
         dtc.selector_ar(np.array([0, 5, 3], np.int32), 2, 1)
+
+
+# ------------------------------------------------------------------ B200 Selector (NEXT-4, reading C26)
+def _units(nbs, split=None):
+    """dtc_format_export unit records: whole-window units of the given block counts, or split pieces
+    (split = list of (window, piece, npieces) per unit)."""
+    out, b = [], 0
+    for k, nb in enumerate(nbs):
+        sid, piece, npc = (-1, 0, 1) if split is None or split[k] is None else (split[k][0], split[k][1], split[k][2])
+        out.append([k, k + 1, b, b + nb, sid, piece, npc, 0])
+        b += nb
+    return np.array(out, dtype=np.int32)
+
+
+def test_b200_simulate_hand_worked():
+    """List scheduling in unit order on S x O slots, earliest-free slot (lowest on ties):
+    1 SM x 2 slots, block 1 ns, no CTA cost: [3,1,2,2,5] -> s0: 3, s1: 1, s1: 3, s0 (tie at 3): 5,
+    s1: 8 -> makespan 8; with cta_ns = 1 every unit costs 1 more: s0 4, s1 2, s1 5, s0 7, s1 11."""
+    m = dtc.make_model(1, 2, 0.0, 1.0, 0.0)
+    assert dtc.selector_simulate(_units([3, 1, 2, 2, 5]), m) == 8.0
+    m = dtc.make_model(1, 2, 1.0, 1.0, 0.0)
+    assert dtc.selector_simulate(_units([3, 1, 2, 2, 5]), m) == 11.0
+
+
+def test_b200_simulate_split_fixup_chain():
+    """The last piece of a window split into np pieces pays fixup_ns x (G + ceil(np/G)),
+    G = np for np <= 4 else ceil(sqrt(np)): 4 pieces of 2 blocks on 4 slots -> 2 + (4 + 1) x 10."""
+    m = dtc.make_model(2, 2, 0.0, 1.0, 10.0)
+    sp = [(0, p, 4) for p in range(4)]
+    assert dtc.selector_simulate(_units([2, 2, 2, 2], sp), m) == 2.0 + 50.0
+    sp9 = [(0, p, 9) for p in range(9)]       # G = 3 -> chain 3 + 3 = 6
+    m1 = dtc.make_model(9, 1, 0.0, 1.0, 1.0)
+    assert dtc.selector_simulate(_units([1] * 9, sp9), m1) == 1.0 + 6.0
+
+
+def test_b200_plan_closed_forms():
+    """Closed-form cases of the plan.  4096 windows of 8 blocks on 888 slots with a CTA cost of 1e6:
+    U=16 gives 2048 units = 3 waves (3 x (1e6 + 16)), U=64 512 units and U=256 128 units = one wave
+    each (1e6 + 64 and 1e6 + 256) -> U=64.  One 300-block window on one slot: every split finishes
+    at 300 (no CTA cost), ties go to the larger U."""
+    rwo = np.arange(0, 8 * 4096 + 1, 8, dtype=np.int32)
+    r = dtc.selector_plan(rwo, dtc.make_model(148, 6, 1e6, 1.0, 0.0), [16, 64, 256], guided=-1)
+    ms = {p["unit_blocks"]: p["makespan_ns"] for p in r["plans"] if p["makespan_ns"] >= 0}
+    assert ms == {16: 3 * (1e6 + 16), 64: 1e6 + 64, 256: 1e6 + 256}
+    assert r["best"]["unit_blocks"] == 64
+    rwo2 = np.array([0, 300], dtype=np.int32)          # one 300-block window, 1 slot: splitting cannot help
+    r2 = dtc.selector_plan(rwo2, dtc.make_model(1, 1, 0.0, 1.0, 0.0), [16, 512], guided=-1)
+    assert r2["best"]["makespan_ns"] == 300.0 and r2["best"]["unit_blocks"] == 512
