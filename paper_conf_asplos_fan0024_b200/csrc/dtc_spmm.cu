@@ -122,6 +122,9 @@ __device__ __forceinline__ bool fp16_pair(int dt, int i, int nblocks, int bb, in
     return dt == DTC_FP16 && i + 1 < nblocks && bb + i + 1 != next_end && (i + 1) % kFp16PairSpan != 0;
 }
 
+// split-fixup counters per (slot, column group, consumer warp): room for up to 16 consumer warps
+constexpr int kFixupWarps = 16;
+
 struct alignas(16) V16 {
     uint32_t w[4];
 };
@@ -681,12 +684,19 @@ template <int DT, int H> constexpr int pad_aslot() { return pad_aval_bytes<DT, H
 // and for tall windows; with 2 TF32 consumer warps its barrier and the 16 KB of fragments (fewer
 // CTAs per SM) cost more than they save: c3 +13.6%, c5 +7.2%, c4/256 +15%, c3h +6.4%, but
 // c2 -14%, c4/128 -13.5% (profiles/r02_ab_coop.txt).
+// 128-byte column segments per consumer warp: 2 (64 fp32 / 128 fp16 columns); -DDTC_PAD_SEG8_CW=1
+// gives 1 KB-slice CTAs twice the consumer warps with half the columns each (sweeps)
+#ifndef DTC_PAD_SEG8_CW
+#define DTC_PAD_SEG8_CW 2
+#endif
+template <int SEG> constexpr int pad_cw() { return SEG == 8 ? DTC_PAD_SEG8_CW : 2; }
+template <int SL, int SEG> constexpr int pad_consumers() { return SL * SEG / pad_cw<SEG>(); }
 #ifndef DTC_PAD_COOP_FORCE
 #define DTC_PAD_COOP_FORCE -1
 #endif
 template <int DT, int SL, int SEG, int H>
 constexpr bool pad_coop() {
-    return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || SL * SEG / 2 >= 4 || H > 1);
+    return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || pad_consumers<SL, SEG>() >= 4 || H > 1);
 }
 template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
     return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<DT, H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
@@ -700,9 +710,13 @@ constexpr size_t pad_smem_bytes() {
            pad_frag_bytes<DT, SL, SEG, H>() + 128;
 }
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
+#ifndef DTC_PAD_CW1_REGS
+#define DTC_PAD_CW1_REGS 72
+#endif
 template <int DT, int SL, int H = 1>
 constexpr int pad_maxregs() {
     if (H > 1) return SL >= 2 ? 112 : 128;   // two 16-row accumulator tiles per thread
+    if (DTC_PAD_SEG8_CW == 1 && DT == DTC_TF32) return DTC_PAD_CW1_REGS;
 #ifdef DTC_PAD_MAXREGS
     return DTC_PAD_MAXREGS;
 #else
@@ -746,7 +760,8 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
 template <int DT, int SL, int SEG, bool VEC, int H, bool TRACE = false>
 // (min-blocks form of the register cap: measured 8-13% faster than __maxnreg__ with the same cap,
 // profiles/r02_ab_launch_bounds.txt)
-__global__ void __launch_bounds__((SL * SEG / 2 + 1) * 32, 65536 / ((SL * SEG / 2 + 1) * 32 * pad_maxregs<DT, SL, H>()))
+__global__ void __launch_bounds__((pad_consumers<SL, SEG>() + 1) * 32,
+                                  65536 / ((pad_consumers<SL, SEG>() + 1) * 32 * pad_maxregs<DT, SL, H>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
@@ -764,10 +779,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         tr[1] = smid();
         tr[2] = gtimer();
     }
-    constexpr int CW = 2;                      // 128-byte segments per consumer warp
+    constexpr int CW = pad_cw<SEG>();          // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
-    constexpr int WPS = SEG / 2;               // consumer warps per slice
+    constexpr int WPS = SEG / CW;              // consumer warps per slice
     constexpr int ROWB = pad_row_bytes<SEG>(), ODD = pad_odd_off<SEG>(), SLB = pad_slice_bytes<SEG>();
     constexpr int STAGE = SL * SLB;
     constexpr int SLICE_COLS = SEG * COLW1;    // 128 / 256 fp32 or 256 / 512 fp16 columns per slice
@@ -1245,8 +1260,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (!split) {
             while (cur < u.we) { store_window(cur, true); ++cur; }
         } else {
-            split_fixup_h<H, NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * 8 + warp,
-                                                  (int64_t)gridDim.y * 8, C, ldc, M, N, g, lane, base, hoff, rowmap);
+            split_fixup_h<H, NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * kFixupWarps + warp,
+                                                  (int64_t)gridDim.y * kFixupWarps, C, ldc, M, N, g, lane, base, hoff,
+                                                  rowmap);
         }
         gi0 += nblocks;
         gc0 += (nblocks + BATCH - 1) / BATCH;
@@ -1413,7 +1429,7 @@ static cudaError_t lpt_units(dtc_format* h, cudaStream_t s) {
 template <int DT, int SL, int SEG, bool VEC, int H>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     constexpr size_t smem = pad_smem_bytes<SL, SEG, H, DT>();
-    constexpr int threads = (SL * SEG / 2 + 1) * 32;
+    constexpr int threads = (pad_consumers<SL, SEG>() + 1) * 32;
     static KernelState ks;
     const int per_sm = kernel_setup(k_spmm_pad<DT, SL, SEG, VEC, H>, threads, smem, ks, a.h->device);
     if (per_sm < 0) {
@@ -1503,7 +1519,8 @@ int pad_occupancy(int dtype, int64_t N, int window_h) {
         if (smem > 48 * 1024 &&
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
             return -1;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, kern, (sl * seg / 2 + 1) * 32, smem) != cudaSuccess) return -1;
+        const int thr = (sl * seg / (seg == 8 ? pad_cw<8>() : pad_cw<4>()) + 1) * 32;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, kern, thr, smem) != cudaSuccess) return -1;
         return v;
     };
 #define DTC_OCC(DT, H)                                                                                              \
@@ -1604,7 +1621,7 @@ int spmm_launch(dtc_format* h, const void* B, int64_t N, int64_t ldb, float* C, 
     const int64_t npad = gy64 * cta_cols;
     if (h->num_split > 0) {
         // split fixup counters per (slot, column group, consumer warp), self-resetting
-        const int64_t ncnt = h->num_slots * (int64_t)gy * 8;
+        const int64_t ncnt = h->num_slots * (int64_t)gy * kFixupWarps;
         if (ncnt > h->counters_len) {
             dfree(h->counters, s);
             h->counters_len = 0;
