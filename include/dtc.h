@@ -168,6 +168,18 @@ int dtc_spmm(dtc_handle_t h, const void* B, int64_t N, int64_t ldb, float* C, in
 int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
                   int64_t ldc, void* stream);
 
+/* Streaming variant of dtc_spmm_host for a sequence of products with the same A (e.g. GNN inference
+ * over many feature batches): enqueues the copy-in of B_host, the kernel and the copy-out of C
+ * (or zero-copy C, as above) and returns WITHOUT waiting.  The library keeps two device staging sets:
+ * call j's copy-in waits, on the device, only for call j-2's kernel, so the copy-in of call j+1
+ * overlaps the kernel of call j and the copy-out of call j-1 (PCIe is full duplex).  B_host must not
+ * change and C_host must not be read until dtc_spmm_host_wait(h) returns.  Each call computes
+ * exactly what dtc_spmm computes.  Errors: as dtc_spmm_host (checked at enqueue). */
+int dtc_spmm_host_async(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
+                        int64_t ldc, void* stream);
+/* Wait for every dtc_spmm_host_async call enqueued on h.  Errors: INVALID, CUDA. */
+int dtc_spmm_host_wait(dtc_handle_t h);
+
 /* Number of kernels dtc_spmm launches per call (for launch accounting). */
 int dtc_spmm_launches_per_call(void);
 

@@ -93,6 +93,8 @@ def lib():
             L.dtc_spmm.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_host.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
             L.dtc_spmm_launches_per_call.argtypes = []
+            L.dtc_spmm_host_async.argtypes = [_vp, _vp, _i64, _i64, _vp, _i64, _vp]
+            L.dtc_spmm_host_wait.argtypes = [_vp]
             L.dtc_format_set_option.argtypes = [_vp, _i32, _i64]
             L.dtc_format_get_option.argtypes = [_vp, _i32, _vp]
             L.dtc_format_set_trace.argtypes = [_vp, _vp, _i64]
@@ -380,6 +382,24 @@ class Format:
             raise TypeError(f"C_host must be float32 of shape ({self.M}, {N}), got {cdt} {(M, Nc)}")
         _check(lib().dtc_spmm_host(self._h, bp, N, ldb, cp, ldc, _stream_ptr(stream)), "dtc_spmm_host")
         return C_host
+
+    def spmm_host_async(self, B_host, C_host, stream=None):
+        """Streaming C_host = A @ B_host (dtc_spmm_host_async): returns at once; consecutive calls
+        overlap their copies with the previous kernel.  Keep B_host unchanged and do not read C_host
+        until wait()."""
+        bp, (K, N), ldb, bdt = _host_ptr(B_host, "B_host")
+        want = np.float16 if self.dtype == "fp16" else np.float32
+        if bdt != np.dtype(want) or K != self.K:
+            raise TypeError(f"B_host must be {np.dtype(want)} with K = {self.K} rows")
+        cp, (M, Nc), ldc, cdt = _host_ptr(C_host, "C_host")
+        if cdt != np.dtype(np.float32) or (M, Nc) != (self.M, N):
+            raise TypeError(f"C_host must be float32 of shape ({self.M}, {N})")
+        _check(lib().dtc_spmm_host_async(self._h, bp, N, ldb, cp, ldc, _stream_ptr(stream)), "dtc_spmm_host_async")
+        return C_host
+
+    def wait(self):
+        """Wait for every spmm_host_async call of this handle (dtc_spmm_host_wait)."""
+        _check(lib().dtc_spmm_host_wait(self._h), "dtc_spmm_host_wait")
 
     def close(self):
         if self._h is not None and self._h.value:

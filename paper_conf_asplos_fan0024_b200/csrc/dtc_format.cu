@@ -490,6 +490,14 @@ static void free_format(dtc_format* h, cudaStream_t s) {
     dfree(h->vals, s); dfree(h->mask, s); dfree(h->units, s); dfree(h->counters, s); dfree(h->ws, s);
     for (auto& e : h->hev) if (e) { cudaEventDestroy(e); e = nullptr; }
     for (auto& hs : h->hstream) if (hs) { cudaStreamDestroy(hs); hs = nullptr; }
+    for (int k = 0; k < 2; ++k) {
+        dfree(h->as_B[k], s); dfree(h->as_C[k], s);
+        if (h->as_ev_in[k]) cudaEventDestroy(h->as_ev_in[k]);
+        if (h->as_ev_kernel[k]) cudaEventDestroy(h->as_ev_kernel[k]);
+        if (h->as_ev_out[k]) cudaEventDestroy(h->as_ev_out[k]);
+    }
+    if (h->as_in) cudaStreamDestroy(h->as_in);
+    if (h->as_out) cudaStreamDestroy(h->as_out);
     dfree(h->stage_B, s); dfree(h->stage_C, s); dfree(h->rowmap, s); dfree(h->gemm_ws, s); dfree(h->uctr, s); dfree(h->units_lpt, s); dfree(h->ufirst, s);
 }
 

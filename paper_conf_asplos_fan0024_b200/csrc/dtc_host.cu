@@ -164,6 +164,122 @@ extern "C" int dtc_spmm_host(dtc_handle_t h, const void* B_host, int64_t N, int6
     return rc;
 }
 
+// ------------------------------------------------------------ streaming host API
+// Call j uses staging slot j & 1: its copy-in waits (on the device) for call j-2's kernel to have
+// read that slot's B, its kernel for call j-2's copy-out to have drained that slot's C; nothing
+// waits on the host.  So consecutive calls overlap: copy-in of j+1 || kernel of j || copy-out of
+// j-1 (PCIe is full duplex).  Zero-copy C (pinned mapped C_host, format larger than B) as in
+// dtc_spmm_host.  Every call computes exactly what dtc_spmm computes.
+static int spmm_host_async_impl(dtc_format* h, const void* B_host, int64_t N, int64_t ldb, float* C_host, int64_t ldc,
+                                cudaStream_t s) {
+    const int elt = elt_size(h->dtype);
+    const size_t bbytes = (size_t)std::max<int64_t>(h->K, 1) * N * elt;
+    const size_t cbytes = (size_t)std::max<int64_t>(h->M, 1) * N * sizeof(float);
+    const int slot = (int)(h->as_seq & 1);
+    float* Czc = nullptr;
+    {
+        bool zc = format_bytes(h, elt) > (double)bbytes && bbytes + cbytes >= ((size_t)8 << 20);
+        if (h->opt.host_zc >= 0) zc = h->opt.host_zc > 0;
+        if (zc) {
+            cudaPointerAttributes at{};
+            if (cudaPointerGetAttributes(&at, C_host) != cudaSuccess) cudaGetLastError();
+            else if (at.type == cudaMemoryTypeHost && at.devicePointer) Czc = reinterpret_cast<float*>(at.devicePointer);
+        }
+    }
+    h->last_host_mode = 2 + (Czc ? 1 : 0);
+    if (!h->as_in) DTC_CUDA(cudaStreamCreateWithFlags(&h->as_in, cudaStreamNonBlocking));
+    if (!h->as_out) DTC_CUDA(cudaStreamCreateWithFlags(&h->as_out, cudaStreamNonBlocking));
+    for (int k = 0; k < 2; ++k) {
+        if (!h->as_ev_in[k]) DTC_CUDA(cudaEventCreateWithFlags(&h->as_ev_in[k], cudaEventDisableTiming));
+        if (!h->as_ev_kernel[k]) DTC_CUDA(cudaEventCreateWithFlags(&h->as_ev_kernel[k], cudaEventDisableTiming));
+        if (!h->as_ev_out[k]) DTC_CUDA(cudaEventCreateWithFlags(&h->as_ev_out[k], cudaEventDisableTiming));
+    }
+    // (re)size this slot's staging: freed in stream order after the slot's previous kernel / copy-out
+    if (bbytes > h->as_B_bytes[slot] || (!Czc && cbytes > h->as_C_bytes[slot])) {
+        DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_kernel[slot], 0));
+        DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_out[slot], 0));
+    }
+    if (bbytes > h->as_B_bytes[slot]) {
+        dfree(h->as_B[slot], s);
+        h->as_B_bytes[slot] = 0;
+        uint8_t* b = nullptr;
+        int rc = dalloc(&b, bbytes, s);
+        if (rc) return rc;
+        h->as_B[slot] = b;
+        h->as_B_bytes[slot] = bbytes;
+    }
+    if (!Czc && cbytes > h->as_C_bytes[slot]) {
+        dfree(h->as_C[slot], s);
+        h->as_C_bytes[slot] = 0;
+        int rc = dalloc(&h->as_C[slot], cbytes / sizeof(float), s);
+        if (rc) return rc;
+        h->as_C_bytes[slot] = cbytes;
+    }
+    // copy-in after everything already queued on s (allocations) and after call j-2's kernel
+    cudaEvent_t ev_q = h->as_ev_in[slot];
+    DTC_CUDA(cudaEventRecord(ev_q, s));
+    DTC_CUDA(cudaStreamWaitEvent(h->as_in, ev_q, 0));
+    DTC_CUDA(cudaStreamWaitEvent(h->as_in, h->as_ev_kernel[slot], 0));
+    if (h->K > 0)
+        DTC_CUDA(cudaMemcpy2DAsync(h->as_B[slot], N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice,
+                                   h->as_in));
+    DTC_CUDA(cudaEventRecord(h->as_ev_in[slot], h->as_in));
+    DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_in[slot], 0));
+    if (Czc) {
+        int rc = spmm_launch(h, h->as_B[slot], N, N, Czc, ldc, s);
+        if (rc) return rc;
+        DTC_CUDA(cudaEventRecord(h->as_ev_kernel[slot], s));
+        DTC_CUDA(cudaEventRecord(h->as_ev_out[slot], s));
+    } else {
+        DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_out[slot], 0));   // call j-2's copy-out drained this C slot
+        int rc = spmm_launch(h, h->as_B[slot], N, N, h->as_C[slot], N, s);
+        if (rc) return rc;
+        DTC_CUDA(cudaEventRecord(h->as_ev_kernel[slot], s));
+        DTC_CUDA(cudaStreamWaitEvent(h->as_out, h->as_ev_kernel[slot], 0));
+        if (h->M > 0)
+            DTC_CUDA(cudaMemcpy2DAsync(C_host, ldc * sizeof(float), h->as_C[slot], N * sizeof(float), N * sizeof(float),
+                                       h->M, cudaMemcpyDeviceToHost, h->as_out));
+        DTC_CUDA(cudaEventRecord(h->as_ev_out[slot], h->as_out));
+    }
+    h->as_last = s;
+    ++h->as_seq;
+    return DTC_OK;
+}
+
+extern "C" int dtc_spmm_host_async(dtc_handle_t h, const void* B_host, int64_t N, int64_t ldb, float* C_host,
+                                   int64_t ldc, void* stream) {
+    if (!h || !C_host || (!B_host && h->K > 0)) { set_error("null argument"); return DTC_ERR_INVALID; }
+    if (N < 1 || ldb < N || ldc < N) { set_error("bad N/ldb/ldc"); return DTC_ERR_INVALID; }
+    int prev = -1;
+    if (cudaGetDevice(&prev) != cudaSuccess) { cudaGetLastError(); set_error("no CUDA device"); return DTC_ERR_CUDA; }
+    if (prev != h->device && cudaSetDevice(h->device) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("cannot select the handle's device %d", h->device);
+        return DTC_ERR_CUDA;
+    }
+    const int rc = spmm_host_async_impl(h, B_host, N, ldb, C_host, ldc, (cudaStream_t)stream);
+    if (prev != h->device) cudaSetDevice(prev);
+    return rc;
+}
+
+extern "C" int dtc_spmm_host_wait(dtc_handle_t h) {
+    if (!h) { set_error("null handle"); return DTC_ERR_INVALID; }
+    int prev = -1;
+    if (cudaGetDevice(&prev) != cudaSuccess) { cudaGetLastError(); set_error("no CUDA device"); return DTC_ERR_CUDA; }
+    if (prev != h->device) cudaSetDevice(h->device);
+    cudaError_t e = cudaSuccess;
+    auto sync = [&](cudaStream_t st) {
+        const cudaError_t e2 = cudaStreamSynchronize(st);
+        if (e == cudaSuccess) e = e2;
+    };
+    if (h->as_in) sync(h->as_in);
+    if (h->as_seq > 0) sync(h->as_last);   // the compute stream of the last call (may be the legacy stream)
+    if (h->as_out) sync(h->as_out);
+    if (prev != h->device) cudaSetDevice(prev);
+    if (e != cudaSuccess) return cuda_fail(e, "dtc_spmm_host_wait", __FILE__, __LINE__);
+    return DTC_OK;
+}
+
 extern "C" int dtc_format_set_option(dtc_handle_t h, int32_t option, int64_t value) {
     if (!h) { set_error("null handle"); return DTC_ERR_INVALID; }
     auto bad = [&]() {

@@ -72,6 +72,14 @@ struct dtc_format {
     // per-chunk events, created on first use
     cudaStream_t hstream[2] = {nullptr, nullptr};
     cudaEvent_t hev[2 * 16 + 1] = {};
+    // streaming host API (dtc_spmm_host_async): two staging sets, copy streams, per-slot events
+    void* as_B[2] = {nullptr, nullptr};
+    size_t as_B_bytes[2] = {0, 0};
+    float* as_C[2] = {nullptr, nullptr};
+    size_t as_C_bytes[2] = {0, 0};
+    cudaStream_t as_in = nullptr, as_out = nullptr, as_last = nullptr;
+    cudaEvent_t as_ev_in[2] = {}, as_ev_kernel[2] = {}, as_ev_out[2] = {};
+    int64_t as_seq = 0;
     // optional row map (row of the condensed matrix -> row of C), from dtc_build_opts_t.row_perm
     int32_t* rowmap = nullptr;
     // launch options and diagnostics

@@ -296,3 +296,29 @@ def test_binding_rejects_mismatched_buffers():
     f16 = build(M, K, rp, ci, v, dtype="fp16")
     with pytest.raises(TypeError):
         f16.spmm_host(good)
+
+
+@pytest.mark.parametrize("zc", [0, 1])
+@pytest.mark.parametrize("dtype,N", [("tf32", 128), ("fp16", 96), ("tf32", 37)])
+def test_host_async_stream_matches_device(zc, dtype, N):
+    """dtc_spmm_host_async: a stream of 5 products with different B (alternating pinned host buffers,
+    as a serving loop would), waited once at the end; every C equals dtc_spmm bit for bit."""
+    import torch
+    M, K = 3000, 2500
+    rp, ci = datagen.random_csr(M, K, 0.01, N + 3)
+    v = datagen.uniform(N, 7, len(ci))
+    f = build(M, K, rp, ci, v, dtype=dtype, options={"host_zero_copy": zc})
+    Bs, refs, Cs = [], [], []
+    for j in range(5):
+        B = datagen.uniform(N + j, 8, K * N).reshape(K, N)
+        if dtype == "fp16":
+            B = B.astype(np.float16)
+        Bs.append(torch.from_numpy(B).pin_memory())
+        refs.append(spmm(f, B))
+        Cs.append(torch.full((M, N), float("nan"), dtype=torch.float32).pin_memory())
+    for j in range(5):
+        f.spmm_host_async(Bs[j], Cs[j])
+    f.wait()
+    for j in range(5):
+        assert np.array_equal(Cs[j].numpy(), refs[j])
+    assert f.get_option("last_host_mode") == 2 + zc
