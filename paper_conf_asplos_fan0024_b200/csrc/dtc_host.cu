@@ -195,7 +195,8 @@ static int spmm_host_async_impl(dtc_format* h, const void* B_host, int64_t N, in
         if (!h->as_ev_out[k]) DTC_CUDA(cudaEventCreateWithFlags(&h->as_ev_out[k], cudaEventDisableTiming));
     }
     // (re)size this slot's staging: freed in stream order after the slot's previous kernel / copy-out
-    if (bbytes > h->as_B_bytes[slot] || (!Czc && cbytes > h->as_C_bytes[slot])) {
+    const bool realloc = bbytes > h->as_B_bytes[slot] || (!Czc && cbytes > h->as_C_bytes[slot]);
+    if (realloc) {
         DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_kernel[slot], 0));
         DTC_CUDA(cudaStreamWaitEvent(s, h->as_ev_out[slot], 0));
     }
@@ -215,10 +216,13 @@ static int spmm_host_async_impl(dtc_format* h, const void* B_host, int64_t N, in
         if (rc) return rc;
         h->as_C_bytes[slot] = cbytes;
     }
-    // copy-in after everything already queued on s (allocations) and after call j-2's kernel
-    cudaEvent_t ev_q = h->as_ev_in[slot];
-    DTC_CUDA(cudaEventRecord(ev_q, s));
-    DTC_CUDA(cudaStreamWaitEvent(h->as_in, ev_q, 0));
+    // copy-in after call j-2's kernel (it read this slot's B) -- and, when this call (re)allocated the
+    // slot, after the stream-ordered allocation on s; otherwise NOT after s's queue, so the copy-in
+    // of call j+1 overlaps the kernel of call j
+    if (realloc) {
+        DTC_CUDA(cudaEventRecord(h->as_ev_in[slot], s));
+        DTC_CUDA(cudaStreamWaitEvent(h->as_in, h->as_ev_in[slot], 0));
+    }
     DTC_CUDA(cudaStreamWaitEvent(h->as_in, h->as_ev_kernel[slot], 0));
     if (h->K > 0)
         DTC_CUDA(cudaMemcpy2DAsync(h->as_B[slot], N * elt, B_host, ldb * elt, N * elt, h->K, cudaMemcpyHostToDevice,
