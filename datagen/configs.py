@@ -3,7 +3,7 @@
 Each config is a generator recipe (pattern + value kind + N + dtype + seeds),
 not data.  Shapes follow the paper's datasets (Table 1) and
 the public OGB/Planetoid statistics named in SURVEY.md §8(d); p_local was
-calibrated once (tools/calibrate.py) so that MeanNnzTC lands near the target
+calibrated once (tests/tools/calibrate.py) so that MeanNnzTC lands near the target
 (Table 2) and then frozen here.
 """
 from __future__ import annotations

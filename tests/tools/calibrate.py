@@ -2,12 +2,12 @@
 
 Run once; the resulting p_local values are frozen in datagen/configs.py.
 Uses only datagen/ and the oracle's condensation count (oracle/).
-    python tools/calibrate.py c1 c2 c3 c5
+    python tests/tools/calibrate.py c1 c2 c3 c5
 """
 import sys
 import os
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 
 from datagen import configs  # noqa: E402
 import oracle  # noqa: E402

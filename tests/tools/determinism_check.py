@@ -1,7 +1,7 @@
 """Determinism + exactness check of dtc_spmm on a config with integer inputs (three runs vs O1 on the
 first 200k rows) -- the check that found the early A-slot release race; usage: determinism_check.py c4 256 [U]."""
 import sys, os, numpy as np, torch
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 import datagen, oracle
 from datagen import configs
 import paper_conf_asplos_fan0024_b200 as dtc
