@@ -1502,7 +1502,10 @@ PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes) {
     if (slice_bytes == 1024 && (N * elt) % 8 == 0) g.seg = 8;
     const int64_t slice_cols = g.seg * 128 / elt;
     const int64_t nsl = (N + slice_cols - 1) / slice_cols;
-    g.slices = nsl >= 2 ? 2 : 1;
+#ifndef DTC_PAD_MAX_SLICES
+#define DTC_PAD_MAX_SLICES 2
+#endif
+    g.slices = nsl >= 2 && DTC_PAD_MAX_SLICES >= 2 ? 2 : 1;
     g.cta_cols = g.slices * slice_cols;
     return g;
 }
