@@ -48,6 +48,30 @@ static int nccl_fail(ncclResult_t r, const char* what) {
         if (_r != ncclSuccess) return ::dtc::nccl_fail(_r, #call);  \
     } while (0)
 
+// pack B(:, columns [off, off + w)) (row pitch ldb bytes) into a contiguous K x w block: one pass at
+// HBM rate (a pitched cudaMemcpy2D of narrow rows runs far below it); V = bytes per access
+template <class V>
+__global__ void k_pack_cols(const uint8_t* __restrict__ B, int64_t ldb, int64_t off, int64_t w, int64_t K,
+                            uint8_t* __restrict__ dst) {
+    const int64_t per_row = w / (int64_t)sizeof(V), n = per_row * K;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / per_row, k = i - r * per_row;
+        reinterpret_cast<V*>(dst + r * w)[k] = *reinterpret_cast<const V*>(B + r * ldb + off + k * (int64_t)sizeof(V));
+    }
+}
+
+static cudaError_t pack_cols(const void* B, int64_t ldb, int64_t off, int64_t w, int64_t K, void* dst, cudaStream_t s) {
+    const uintptr_t a = (uintptr_t)B | (uintptr_t)dst | (uintptr_t)ldb | (uintptr_t)off | (uintptr_t)w;
+    const unsigned grid = 148 * 8;
+    if (a % 16 == 0)
+        k_pack_cols<uint4><<<grid, 256, 0, s>>>((const uint8_t*)B, ldb, off, w, K, (uint8_t*)dst);
+    else if (a % 4 == 0)
+        k_pack_cols<uint32_t><<<grid, 256, 0, s>>>((const uint8_t*)B, ldb, off, w, K, (uint8_t*)dst);
+    else
+        k_pack_cols<uint8_t><<<grid, 256, 0, s>>>((const uint8_t*)B, ldb, off, w, K, (uint8_t*)dst);
+    return cudaGetLastError();
+}
+
 __global__ void k_rebase(const int32_t* __restrict__ in, int32_t* __restrict__ out, int64_t n, int32_t base) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = in[i] - base;
@@ -205,8 +229,7 @@ extern "C" int dtc_spmm_dist(dtc_dist_t d, void* B, int32_t root, int64_t N, flo
         uint8_t* bj = d->stage + (size_t)d->K * cb[j] * elt;
         if (d->K > 0) {
             if (d->rank == root)   // pack the chunk's columns (strided) into the contiguous chunk buffer
-                DTC_CUDA(cudaMemcpy2DAsync(bj, nc * elt, (const uint8_t*)B + cb[j] * elt, N * elt, nc * elt, d->K,
-                                           cudaMemcpyDeviceToDevice, cs));
+                DTC_CUDA(pack_cols(B, N * elt, cb[j] * elt, nc * elt, d->K, bj, cs));
             DTC_NCCL(ncclBroadcast(bj, bj, (size_t)(d->K * nc), bt, root, d->comm, cs));
         }
         DTC_CUDA(cudaEventRecord(d->ev_chunk[j], cs));
