@@ -140,6 +140,28 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+// the same on a shared-memory address (the kernel keeps every barrier address relative to one base
+// register instead of re-deriving a generic -> shared conversion per use)
+__device__ __forceinline__ void mbar_init(uint32_t bar, int count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n"
@@ -651,8 +673,9 @@ template <int SEG> constexpr int pad_tx_bytes() { return 8 * pad_row_bytes<SEG>(
 static_assert(pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16, "row pitch must be 16 mod 128");
 static_assert(pad_row_bytes<4>() % 8 == 0 && pad_row_bytes<8>() % 8 == 0, "row pitch: whole 8-byte elements");
 // B ring depth (stages of SL slices); measured flat between 3 and 6 once the A side is staged
-// (profiles/r01_design_evidence.md), deeper rings only cost CTAs per SM.  -DDTC_PAD_STAGES=k
-// overrides for sweeps.
+// (profiles/r01_design_evidence.md), and 6-10 stages with 8-block A batches 4-22% slower than 4
+// (profiles/r02_ab_issue.txt): deeper rings only cost CTAs per SM.  -DDTC_PAD_STAGES=k overrides
+// for sweeps.
 template <int SL>
 constexpr int pad_stages() {
 #ifdef DTC_PAD_STAGES
@@ -667,18 +690,46 @@ constexpr int pad_stages() {
 constexpr int kPadBatch = 16;
 static_assert(kPadBatch % kFp16PairSpan == 0, "FP16 pairs never straddle an A batch");
 // per-unit side record for the first batch (DTC_OPT_FIRST_RECORDS): kPadBatch x 8 SparseAtoB ids
-// (-1 past the unit), TCOffset[bb], TCOffset[bb + min(kPadBatch, nb)], end of the first window, pad
+// (-1 past the unit), TCOffset[bb], TCOffset[bb + min(kPadBatch, nb)], end of the first window,
+// TCOffset[bb + min(kPadBatch / 2, nb)] -- one record serves kernels with A batches of 16 or 8 blocks
 constexpr int kFirstRec = kPadBatch * 8 + 4;
 static_assert((kFirstRec * 4) % 16 == 0, "int4 loads of the side record");
+// Per-geometry tuning (measured on one box, profiles/r02_ab_issue.txt):
+//  * "slim" CTAs -- TF32, one slice, 16-row windows (c3, c2, c4 N <= 128): A batches of 8 blocks and a
+//    96-register cap fit 4 CTAs per SM instead of 3 on c3 (smem 51 KB, 20 warps): c3 +6.5-6.9%, c4
+//    N=64/128 +4%, c2 -0.3%.  The consumers' ~70
+//    instructions per block run at ~7 cycles each, so more resident warps, not a deeper B ring
+//    (6-10 stages measured 4-22% slower), is what raises the block rate.
+//  * FP16 and two-slice CTAs (c3h, c5): the producer issues the gathers of 2 TC blocks per pass
+//    (G = 2; its per-block bookkeeping halves): c3h +4%, c5 +1%.  G <= R - 1: a consumer holding an
+//    FP16 pair's first stage waits for the second, which a G = R group would never issue.
+// -DDTC_PAD_TF32_BATCH / DTC_PAD_MAXREGS / DTC_PAD_ISSUE / DTC_PAD_STAGES override every geometry
+// (sweeps).
+template <int DT, int SL, int SEG, int H> constexpr bool pad_slim() { return DT == DTC_TF32 && H == 1 && SL == 1; }
+template <int DT, int SL, int SEG, int H>
+constexpr int pad_issue() {
+#ifdef DTC_PAD_ISSUE
+    return DTC_PAD_ISSUE;
+#else
+    return (DT == DTC_FP16 || SL == 2) ? 2 : 1;
+#endif
+}
+static_assert(pad_issue<DTC_FP16, 2, 8, 1>() <= pad_stages<2>() - 1 && pad_issue<DTC_FP16, 1, 4, 1>() <= pad_stages<1>() - 1,
+              "issue group <= ring depth - 1");
 // A batch slot for windows of H x 16 rows: values (<= batch x 128H x 4 B + 16, 128-aligned), then
 // one 16H-byte occupancy mask per block
 // (tall windows take batches of kPadBatch / H blocks, so a batch slot is the same size for every H)
-#ifndef DTC_PAD_TF32_BATCH
-#define DTC_PAD_TF32_BATCH 16
+template <int DT, int SL, int SEG, int H> constexpr int pad_batch() {
+#ifdef DTC_PAD_TF32_BATCH
+    if (DT == DTC_TF32) return DTC_PAD_TF32_BATCH / H;
 #endif
-template <int DT, int H> constexpr int pad_batch() { return (DT == DTC_TF32 ? DTC_PAD_TF32_BATCH : kPadBatch) / H; }
-template <int DT, int H> constexpr int pad_aval_bytes() { return pad_batch<DT, H>() * 512 * H + 128; }
-template <int DT, int H> constexpr int pad_aslot() { return pad_aval_bytes<DT, H>() + pad_batch<DT, H>() * 16 * H; }
+    return pad_slim<DT, SL, SEG, H>() ? kPadBatch / 2 : kPadBatch / H;
+}
+static_assert(kPadBatch % 8 == 0, "first records hold the A range of the first 8 and 16 blocks");
+template <int DT, int SL, int SEG, int H> constexpr int pad_aval_bytes() { return pad_batch<DT, SL, SEG, H>() * 512 * H + 128; }
+template <int DT, int SL, int SEG, int H> constexpr int pad_aslot() {
+    return pad_aval_bytes<DT, SL, SEG, H>() + pad_batch<DT, SL, SEG, H>() * 16 * H;
+}
 // Cooperative A expansion (consumers decode each block once into shared memory) pays where a
 // CTA has >= 4 consumer warps (each would otherwise decode every block), for FP16 (block pairs),
 // and for tall windows; with 2 TF32 consumer warps its barrier and the 16 KB of fragments (fewer
@@ -699,28 +750,28 @@ constexpr bool pad_coop() {
     return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || pad_consumers<SL, SEG>() >= 4 || H > 1);
 }
 template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
-    return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<DT, H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
+    return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<DT, SL, SEG, H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
 }
 // raw A batch slots (double buffered; a third slot would let the producer run a batch further ahead
 // but costs a CTA per SM on c3: 8.59 -> 6.88 TFLOP/s measured, profiles/r02_ab_coop_slots.txt)
 template <int DT, int SL, int SEG, int H> constexpr int pad_aslots() { return 2; }
 template <int SL, int SEG, int H = 1, int DT = DTC_TF32>
 constexpr size_t pad_smem_bytes() {
-    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<DT, H>() +
-           pad_frag_bytes<DT, SL, SEG, H>() + 128;
+    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<DT, SL, SEG, H>() +
+           pad_frag_bytes<DT, SL, SEG, H>() + 128 + 256;   // + alignment slack + mbarriers
 }
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
 #ifndef DTC_PAD_CW1_REGS
 #define DTC_PAD_CW1_REGS 72
 #endif
-template <int DT, int SL, int H = 1>
+template <int DT, int SL, int SEG, int H>
 constexpr int pad_maxregs() {
     if (H > 1) return SL >= 2 ? 112 : 128;   // two 16-row accumulator tiles per thread
     if (DTC_PAD_SEG8_CW == 1 && DT == DTC_TF32) return DTC_PAD_CW1_REGS;
 #ifdef DTC_PAD_MAXREGS
     return DTC_PAD_MAXREGS;
 #else
-    return DT == DTC_FP16 ? 128 : 104;
+    return DT == DTC_FP16 ? 128 : (pad_slim<DT, SL, SEG, H>() ? 96 : 104);
 #endif
 }
 
@@ -761,7 +812,7 @@ template <int DT, int SL, int SEG, bool VEC, int H, bool TRACE = false>
 // (min-blocks form of the register cap: measured 8-13% faster than __maxnreg__ with the same cap,
 // profiles/r02_ab_launch_bounds.txt)
 __global__ void __launch_bounds__((pad_consumers<SL, SEG>() + 1) * 32,
-                                  65536 / ((pad_consumers<SL, SEG>() + 1) * 32 * pad_maxregs<DT, SL, H>()))
+                                  65536 / ((pad_consumers<SL, SEG>() + 1) * 32 * pad_maxregs<DT, SL, SEG, H>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
@@ -782,20 +833,26 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     constexpr int CW = pad_cw<SEG>();          // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
+    constexpr int G = pad_issue<DT, SL, SEG, H>();
     constexpr int WPS = SEG / CW;              // consumer warps per slice
     constexpr int ROWB = pad_row_bytes<SEG>(), ODD = pad_odd_off<SEG>(), SLB = pad_slice_bytes<SEG>();
     constexpr int STAGE = SL * SLB;
     constexpr int SLICE_COLS = SEG * COLW1;    // 128 / 256 fp32 or 256 / 512 fp16 columns per slice
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t ring = (smem_u32(smem_raw) + 127u) & ~127u;       // [R][STAGE] B stages
-    constexpr int BATCH = pad_batch<DT, H>();   // TC blocks per A batch
-    constexpr int ASLOT = pad_aslot<DT, H>(), AVAL = pad_aval_bytes<DT, H>(), NA = pad_aslots<DT, SL, SEG, H>();
+    constexpr int BATCH = pad_batch<DT, SL, SEG, H>();   // TC blocks per A batch
+    static_assert(BATCH == kPadBatch || BATCH == kPadBatch / 2, "first records carry the A range of 8 or 16 blocks");
+    constexpr int ASLOT = pad_aslot<DT, SL, SEG, H>(), AVAL = pad_aval_bytes<DT, SL, SEG, H>(), NA = pad_aslots<DT, SL, SEG, H>();
     const uint32_t aring = ring + R * STAGE;                          // [2][ASLOT] A batches
-    __shared__ __align__(8) uint64_t bar_full[R], bar_empty[R], bar_afull[NA], bar_aempty[NA], bar_ufull[2], bar_uempty[2];
-    __shared__ int s_abyte[NA];   // byte offset of the batch's first value inside its A slot (batch c: slot c % NA)
+    __shared__ int s_abyte[NA];   // byte offset of the batch's first value inside its A slot (batch c: slot (uint32_t)c % NA)
     constexpr bool COOP = pad_coop<DT, SL, SEG, H>();
     __shared__ uint8_t s_live[2][BATCH];   // COOP: per block, bit h = sub-tile h has a non-zero
     const uint32_t frags = aring + NA * ASLOT;  // COOP: [2][BATCH][H] lane-major fragments (expand())
+    // mbarriers: full[R], empty[R] (B stages), afull[NA], aempty[NA] (A batches), ufull[2], uempty[2]
+    // (published units) -- after the fragments, 8 bytes each
+    const uint32_t bar_full = frags + pad_frag_bytes<DT, SL, SEG, H>(), bar_empty = bar_full + 8 * R;
+    const uint32_t bar_afull = bar_empty + 8 * R, bar_aempty = bar_afull + 8 * NA;
+    const uint32_t bar_ufull = bar_aempty + 8 * NA, bar_uempty = bar_ufull + 16;
     __shared__ int s_unit[2][10];   // published unit: Unit record, end block of its first window, index (-1 = done)
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -813,16 +870,16 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int ncons = WPS * nsl;               // active consumers
     if (threadIdx.x == 0) {
         for (int i = 0; i < R; ++i) {
-            mbar_init(&bar_full[i], 1);
-            mbar_init(&bar_empty[i], ncons);
+            mbar_init(bar_full + 8u * (i), 1);
+            mbar_init(bar_empty + 8u * (i), ncons);
         }
         for (int i = 0; i < NA; ++i) {
-            mbar_init(&bar_afull[i], 1);
-            mbar_init(&bar_aempty[i], COOP ? 1 : ncons);
+            mbar_init(bar_afull + 8u * (i), 1);
+            mbar_init(bar_aempty + 8u * (i), COOP ? 1 : ncons);
         }
         for (int i = 0; i < 2; ++i) {
-            mbar_init(&bar_ufull[i], 1);
-            mbar_init(&bar_uempty[i], ncons);
+            mbar_init(bar_ufull + 8u * (i), 1);
+            mbar_init(bar_uempty + 8u * (i), ncons);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -893,7 +950,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             rnext.e0 = rnext.e1 = 0;
             if (lane == 0) {
                 rnext.e0 = __ldg(fr + kPadBatch * 8);
-                rnext.e1 = __ldg(fr + kPadBatch * 8 + 1);
+                rnext.e1 = __ldg(fr + kPadBatch * 8 + (BATCH == kPadBatch ? 1 : 3));
             }
             end0 = __ldg(fr + kPadBatch * 8 + 2);
         } else {
@@ -903,53 +960,60 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         int gi0 = 0, gc0 = 0;
         for (int ord = 0;; ++ord) {
             // publish unit ord to the consumers (index -1 = no more units)
-            if (ord >= 2) mbar_wait(&bar_uempty[ord & 1], ((ord >> 1) - 1) & 1);
+            if (ord >= 2) mbar_wait(bar_uempty + 8u * (ord & 1), ((ord >> 1) - 1) & 1);
             if (lane == 0) {
                 int* su = s_unit[ord & 1];
                 su[0] = u.wb; su[1] = u.we; su[2] = u.bb; su[3] = u.be;
                 su[4] = u.split_id; su[5] = u.piece; su[6] = u.npieces; su[7] = u.slot_base;
                 su[8] = end0;
                 su[9] = q0 < num_units ? q0 : -1;
-                mbar_arrive(&bar_ufull[ord & 1]);
+                mbar_arrive(bar_ufull + 8u * (ord & 1));
             }
             if (q0 >= num_units) break;
             const int q2 = draw();   // reserve the unit after next now; its latency hides behind this unit
             const int nblocks = u.be - u.bb;
             for (int i0 = 0; i0 < nblocks; i0 += BATCH) {
-                const int c = gc0 + i0 / BATCH, aslot = c % NA;
+                const int c = gc0 + (uint32_t)i0 / BATCH, aslot = (uint32_t)c % NA;
                 const BatchMeta cur = finish(rnext);
                 rnext = i0 + BATCH < nblocks ? load_raw(u, i0 + BATCH) : load_raw(un, 0);
                 if (i0 == 0) end0n = first_end(un);
                 const int nj = min(BATCH, nblocks - i0);
-                if (c >= NA) mbar_wait(&bar_aempty[aslot], ((c / NA) - 1) & 1);
+                if (c >= NA) mbar_wait(bar_aempty + 8u * (aslot), (((uint32_t)c / NA) - 1) & 1);
                 if (lane == 0) {
                     const int64_t lo = ((int64_t)cur.e0 * ELT) & ~int64_t(15);
                     const int64_t hi = ((int64_t)cur.e1 * ELT + 15) & ~int64_t(15);
                     const uint32_t vbytes = (uint32_t)(hi - lo), mbytes = (uint32_t)nj * 16 * H;
                     const uint32_t dst = aring + aslot * ASLOT;
                     s_abyte[aslot] = (int)((int64_t)cur.e0 * ELT - lo);
-                    mbar_arrive_tx(&bar_afull[aslot], vbytes + mbytes);
+                    mbar_arrive_tx(bar_afull + 8u * (aslot), vbytes + mbytes);
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                                  ::"r"(dst), "l"(reinterpret_cast<const uint8_t*>(avals) + lo), "r"(vbytes),
-                                 "r"(smem_u32(&bar_afull[aslot])) : "memory");
+                                 "r"((bar_afull + 8u * (aslot))) : "memory");
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                                  ::"r"(dst + AVAL), "l"(mask + (int64_t)(u.bb + i0) * H), "r"(mbytes),
-                                 "r"(smem_u32(&bar_afull[aslot])) : "memory");
+                                 "r"((bar_afull + 8u * (aslot))) : "memory");
                 }
-                for (int j = 0; j < nj; ++j) {
-                    const int i = gi0 + i0 + j, s = i % R;
-                    if (i >= R) mbar_wait(&bar_empty[s], ((i / R) - 1) & 1);
-                    if (TRACE && tr && i == 0 && lane == 0) tr[3] = gtimer();
-                    if (lane == 0) mbar_arrive_tx(&bar_full[s], tx);
+                // G blocks per issue: the lane pairs of blocks j0 .. j0+G-1 issue their gather4 ops in ONE
+                // instruction (the producer's instruction rate, not bytes in flight, bounded the gather)
+                for (int j0 = 0; j0 < nj; j0 += G) {
+                    const int gn = min(G, nj - j0);
+                    for (int j = j0; j < j0 + gn; ++j) {
+                        const int i = gi0 + i0 + j;
+                        if (i >= R) mbar_wait(bar_empty + 8u * ((uint32_t)i % R), (((uint32_t)i / R) - 1) & 1);
+                    }
+                    if (TRACE && tr && gi0 + i0 + j0 == 0 && lane == 0) tr[3] = gtimer();
+                    const bool mine = jl >= j0 && jl < j0 + gn;
+                    const int s = (uint32_t)(gi0 + i0 + jl) % R;
+                    if (mine && half == 0) mbar_arrive_tx(bar_full + 8u * (s), tx);
                     __syncwarp();
-                    if (jl == j) {
+                    if (mine) {
                         for (int sl = 0; sl < nsl; ++sl) {
                             const uint32_t dst = ring + s * STAGE + sl * SLB + half * ODD;
                             asm volatile(
                                 "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
                                 " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
                                 "l"(&bmap), "r"(tcol + sl * tslice), "r"(cur.ids.x), "r"(cur.ids.y), "r"(cur.ids.z),
-                                "r"(cur.ids.w), "r"(smem_u32(&bar_full[s]))
+                                "r"(cur.ids.w), "r"((bar_full + 8u * (s)))
                                 : "memory");
                         }
                     }
@@ -1024,9 +1088,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     // rewritten only at batch c+2, after every consumer has passed the barrier of batch c+1.
     constexpr int FSUB = 32 * FW * 4;                      // bytes of one sub-tile's fragments
     auto expand = [&](int c, int nj) {
-        mbar_wait(&bar_afull[c % NA], (c / NA) & 1);
-        const uint32_t slot = aring + (c % NA) * ASLOT;
-        const uint32_t v0 = slot + s_abyte[c % NA], maddr = slot + AVAL;
+        mbar_wait(bar_afull + 8u * ((uint32_t)c % NA), ((uint32_t)c / NA) & 1);
+        const uint32_t slot = aring + ((uint32_t)c % NA) * ASLOT;
+        const uint32_t v0 = slot + s_abyte[(uint32_t)c % NA], maddr = slot + AVAL;
         // value offset of every block of the batch: exclusive warp scan of the blocks' popcounts
         int cnt = 0;
         if (lane < nj)
@@ -1064,10 +1128,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         }
         asm volatile("bar.sync 1, %0;" ::"r"(ncons * 32) : "memory");
     };
-    // this lane's fragments of block i (batch c = gc0 + i / BATCH); live[h] = sub-tile h has a
+    // this lane's fragments of block i (batch c = gc0 + (uint32_t)i / BATCH); live[h] = sub-tile h has a
     // non-zero (warp-uniform)
     auto afrag_coop = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
-        const int j = i % BATCH, c = gc0 + i / BATCH;
+        const int j = (uint32_t)i % BATCH, c = gc0 + (uint32_t)i / BATCH;
         const uint32_t fbase = frags + (c & 1) * (BATCH * H * FSUB) + j * H * FSUB + lane * FW * 4;
         const uint32_t lv = s_live[c & 1][j];
 #pragma unroll
@@ -1087,21 +1151,21 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     // corrupted C on long units -- measured, found with a fragment cross-check; kept late)
     auto release_coop = [&](int i, int gi, int nblocks, int gc0) {
         if (lane == 0) {
-            mbar_arrive(&bar_empty[gi % R]);
-            if (warp == 0 && ((i % BATCH) == BATCH - 1 || i == nblocks - 1)) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) % NA]);
+            mbar_arrive(bar_empty + 8u * ((uint32_t)gi % R));
+            if (warp == 0 && (((uint32_t)i % BATCH) == BATCH - 1 || i == nblocks - 1)) mbar_arrive(bar_aempty + 8u * ((gc0 + (uint32_t)i / BATCH) % NA));
         }
     };
 
     // A batch cursor: the next block's first value (bytes) and the batch's mask array
     uint32_t vaddr = 0, maddr = 0;
-    // S1: the A fragments of block i of the unit (batch c = gc0 + i / BATCH) -- one per 16-row
+    // S1: the A fragments of block i of the unit (batch c = gc0 + (uint32_t)i / BATCH) -- one per 16-row
     // sub-tile h < H -- decoded by every consumer warp for its own columns; blocks in order
     auto afrag_dec = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
-        const int j = i % BATCH, c = gc0 + i / BATCH;
+        const int j = (uint32_t)i % BATCH, c = gc0 + (uint32_t)i / BATCH;
         if (j == 0) {
-            mbar_wait(&bar_afull[c % NA], (c / NA) & 1);
-            const uint32_t slot = aring + (c % NA) * ASLOT;
-            vaddr = slot + s_abyte[c % NA];
+            mbar_wait(bar_afull + 8u * ((uint32_t)c % NA), ((uint32_t)c / NA) & 1);
+            const uint32_t slot = aring + ((uint32_t)c % NA) * ASLOT;
+            vaddr = slot + s_abyte[(uint32_t)c % NA];
             maddr = slot + AVAL;
         }
 #pragma unroll
@@ -1115,9 +1179,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     // release the B stage of CTA block gi and, after a batch's last block, its A slot
     auto release_dec = [&](int i, int gi, int nblocks, int gc0) {
         if (lane == 0) {
-            mbar_arrive(&bar_empty[gi % R]);
-            const int j = i % BATCH;
-            if (j == BATCH - 1 || i == nblocks - 1) mbar_arrive(&bar_aempty[(gc0 + i / BATCH) % NA]);
+            mbar_arrive(bar_empty + 8u * ((uint32_t)gi % R));
+            const int j = (uint32_t)i % BATCH;
+            if (j == BATCH - 1 || i == nblocks - 1) mbar_arrive(bar_aempty + 8u * ((gc0 + (uint32_t)i / BATCH) % NA));
         }
     };
     auto afrag = [&](int i, int gc0, uint32_t (&a)[H][FW], bool (&live)[H]) {
@@ -1133,7 +1197,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     // unit boundary costs no dependent global load.
     int gi0 = 0, gc0 = 0;
     for (int ord = 0;; ++ord) {
-        mbar_wait(&bar_ufull[ord & 1], (ord >> 1) & 1);
+        mbar_wait(bar_ufull + 8u * (ord & 1), (ord >> 1) & 1);
         Unit u;
         int end0, uidx;
         {
@@ -1144,7 +1208,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             uidx = su[9];
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(&bar_uempty[ord & 1]);
+        if (lane == 0) mbar_arrive(bar_uempty + 8u * (ord & 1));
         if (uidx < 0) break;
         const int nblocks = u.be - u.bb;
         const bool split = u.split_id >= 0;
@@ -1171,9 +1235,9 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             next_end = cur < u.we ? e : INT_MAX;
         }
         for (int i = 0; i < nblocks;) {
-            const int gi = gi0 + i, s = gi % R;
+            const int gi = gi0 + i, s = (uint32_t)gi % R;
             if constexpr (COOP)
-                if (i % BATCH == 0) expand(gc0 + i / BATCH, min(BATCH, nblocks - i));
+                if ((uint32_t)i % BATCH == 0) expand(gc0 + (uint32_t)i / BATCH, min(BATCH, nblocks - i));
             // FP16: two TC blocks of one window feed one m16n8k16 (k = block i's 8 columns, then
             // block i+1's -- the k16 A/B fragments are exactly the two k8 fragments side by side)
             const bool pair = fp16_pair(DT, i, nblocks, u.bb, next_end);
@@ -1182,7 +1246,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             afrag(i, gc0, a, live);
             if (pair) afrag(i + 1, gc0, a2, live2);
             // S2/S3: B fragments from the padded stage(s), mma (a sub-tile without non-zeros is skipped)
-            mbar_wait(&bar_full[s], (gi / R) & 1);
+            mbar_wait(bar_full + 8u * (s), ((uint32_t)gi / R) & 1);
             if (TRACE && tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();   // (compiled out unless traced)
             const uint32_t st = ring + s * STAGE;
             if constexpr (DT == DTC_TF32) {
@@ -1196,12 +1260,14 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                     for (int h = 0; h < H; ++h)
                         if (H == 1 || live[h])
 #pragma unroll
+                            // (the B pair {y0, y1} needs register moves before each HMMA; two m16n8k4
+                            // halves avoid them but measured 2-11% slower, profiles/r02_ab_issue.txt)
                             for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[h][cw * NJ1 + jj], a[h], y0[jj & 3], y1[jj & 3]);
                 }
             } else {
                 if (pair) {
-                    const int s2 = (gi + 1) % R;
-                    mbar_wait(&bar_full[s2], ((gi + 1) / R) & 1);
+                    const int s2 = (uint32_t)(gi + 1) % R;
+                    mbar_wait(bar_full + 8u * (s2), ((uint32_t)(gi + 1) / R) & 1);
                     const uint32_t st2 = ring + s2 * STAGE;
 #pragma unroll
                     for (int cw = 0; cw < CW; ++cw) {
@@ -1368,7 +1434,8 @@ static cudaError_t launch_ldg(const LaunchArgs& a, int warps) {
 
 __global__ void k_units_first(int64_t nu, const Unit* __restrict__ units, const int32_t* __restrict__ atob,
                               const int32_t* __restrict__ tco, const int32_t* __restrict__ rwo,
-                              int32_t* __restrict__ out, int batch) {
+                              int32_t* __restrict__ out) {
+    constexpr int batch = kPadBatch;
     for (int64_t q = blockIdx.x; q < nu; q += gridDim.x) {
         const Unit u = units[q];
         const int nb = u.be - u.bb;
@@ -1384,6 +1451,8 @@ __global__ void k_units_first(int64_t nu, const Unit* __restrict__ units, const 
                 v = nb > 0 ? tco[u.bb + min(batch, nb)] : 0;
             } else if (t == kPadBatch * 8 + 2) {
                 v = (u.split_id < 0 && u.wb < u.we) ? rwo[u.wb + 1] : INT_MAX;
+            } else {
+                v = nb > 0 ? tco[u.bb + min(batch / 2, nb)] : 0;
             }
             o[t] = v;
         }
@@ -1398,8 +1467,7 @@ static cudaError_t first_records(dtc_format* h, cudaStream_t s) {
     int32_t* d = nullptr;
     if (dalloc(&d, (size_t)h->num_units * kFirstRec, s) != DTC_OK) return cudaErrorMemoryAllocation;
     k_units_first<<<(unsigned)std::min<int64_t>(h->num_units, 65535), 128, 0, s>>>(
-        h->num_units, h->units, h->atob, h->tco, h->rwo, d,
-        h->dtype == DTC_FP16 ? pad_batch<DTC_FP16, 1>() : (h->window_h == kWindow ? pad_batch<DTC_TF32, 1>() : pad_batch<DTC_TF32, 2>()));
+        h->num_units, h->units, h->atob, h->tco, h->rwo, d);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { dfree(d, s); return e; }
     h->ufirst = d;

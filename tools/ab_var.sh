@@ -4,7 +4,7 @@ mkdir -p gpurun_out; out=gpurun_out/ab_var.txt; : > $out
 B="python bench.py --ncu off --no-cpu --no-cusparse --no-e2e --tca 0 --graphconv 0 --steps 30 --warmup 5"
 run() {
   lab=$1; shift
-  env "$@" | tail -1 | python -c "
+  timeout 400 env "$@" | tail -1 | python -c "
 import json,sys
 d=json.loads(sys.stdin.read())
 rows=[(d['config']['workload'][:3],d['config']['N'],d['value'],d.get('clocks',{}).get('sm_mhz'))]
@@ -14,7 +14,7 @@ for r in rows: print('$lab', *r)
 }
 for rep in 1 2; do
   for v in default ${VARS}; do
-    if [ $v = default ]; then L=""; else L="DTC_LIBRARY=$PWD/build_variants/$v/libdtc.so"; fi
+    if [ $v = default ]; then L=""; else L="DTC_LIBRARY=$PWD/${VDIR:-build_variants}/$v/libdtc.so"; fi
     run $v $L $B --legs ${LEGS:-c2,c4:128,c4:256,c5} 2>/dev/null
   done
 done
