@@ -726,7 +726,10 @@ template <int DT, int SL, int SEG, int H> constexpr int pad_batch() {
     return pad_slim<DT, SL, SEG, H>() ? kPadBatch / 2 : kPadBatch / H;
 }
 static_assert(kPadBatch % 8 == 0, "first records hold the A range of the first 8 and 16 blocks");
-template <int DT, int SL, int SEG, int H> constexpr int pad_aval_bytes() { return pad_batch<DT, SL, SEG, H>() * 512 * H + 128; }
+// (values of one block: at most 16H x 8 elements of the handle's dtype)
+template <int DT, int SL, int SEG, int H> constexpr int pad_aval_bytes() {
+    return pad_batch<DT, SL, SEG, H>() * 128 * H * (DT == DTC_FP16 ? 2 : 4) + 128;
+}
 template <int DT, int SL, int SEG, int H> constexpr int pad_aslot() {
     return pad_aval_bytes<DT, SL, SEG, H>() + pad_batch<DT, SL, SEG, H>() * 16 * H;
 }
