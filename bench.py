@@ -18,7 +18,7 @@ roofline (per leg): `frac` = literal algorithmic bytes (format + 
 M*N*4) / mean kernel time / measured HBM peak; `dram_frac` = DRAM bytes actually moved (ncu
 dram__bytes_read+write of ONE launch of this commit, captured by a subprocess under ncu in this
 run) / mean kernel time / peak; `compulsory_frac` counts every distinct B row once; `gather_frac`
-= gathered B bytes / time / the measured TMA gather4-from-L2 ceiling (profiles/r01_gather_microbench.txt).
+= gathered B bytes / time / the measured TMA gather4-from-L2 peak for the slice width (profiles/r02_gather_issue_sweep.txt).
 `bound_by` names the largest of these fractions.
 
 --impl reference times the FP64 CPU oracle (the only reference this tier has) on the host cores on
@@ -49,8 +49,16 @@ UNIT = "GFLOP/s"
 L2_FLUSH_BYTES = 256 << 20
 HEADLINE = "c3"
 DEFAULT_LEGS = "c2,c3h,c4:64,c4:128,c4:256,c5"
-# TMA tile::gather4 of 2 KB boxes from an L2-resident B, 148 SMs (profiles/r01_gather_microbench.txt)
-GATHER4_L2_CEILING_GBS = 9296.0
+# TMA tile::gather4 peak from an L2-resident B (77 MB), 148 SMs, best over CTAs/SM x gather ops per
+# stage x stages (tools/gather_bw2.py --issue, profiles/r02_gather_issue_sweep.txt), per row-slice
+# width the kernel gathers: 1 KB slices (B rows >= 1 KB) and 512 B slices.  (Round 1's 9.3 TB/s was
+# the rate of one 2-op stage per CTA at 3 CTAs/SM, not the engine's peak.)
+GATHER4_L2_PEAK_GBS = {1024: 18670.0, 512: 12777.0}
+
+
+def gather_peak(N, elt):
+    """the slice width k_spmm_pad gathers for N columns (pad_geometry) -> its measured gather4 peak"""
+    return GATHER4_L2_PEAK_GBS[1024 if (N * elt >= 1024 and (N * elt) % 8 == 0) else 512]
 
 
 def parse_args():
@@ -391,8 +399,8 @@ def run_leg(args, cfg, N, dev, stream, flush, full: bool, cache_dir=None):
                        "compulsory_bytes_per_launch": ab["compulsory"],
                        "compulsory_frac": round(ab["compulsory"] / t / 1e9 / hbm, 4),
                        "gathered_bytes_per_launch": ab["gathered"],
-                       "gather_ceiling_gbs": GATHER4_L2_CEILING_GBS,
-                       "gather_frac": round(ab["gathered"] / t / 1e9 / GATHER4_L2_CEILING_GBS, 4),
+                       "gather_ceiling_gbs": gather_peak(N, elt),
+                       "gather_frac": round(ab["gathered"] / t / 1e9 / gather_peak(N, elt), 4),
                        "kernel_ms_mean": round(kern_ms, 5)}
 
     # ---- e2e through the public API with HOST buffers (pinned): every step copies its B in and

@@ -7,9 +7,6 @@ git log -1 --format=%H > gpurun_out/ev_commit.txt 2>/dev/null
 timeout 900 python bench.py > gpurun_out/ev_bench_default.json 2> gpurun_out/ev_bench_default.err
 timeout 600 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/ev_bench_reference.json 2> gpurun_out/ev_bench_reference.err
 timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > gpurun_out/ev_pytest_gpu.log 2>&1
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_smoke.py > gpurun_out/ev_sanitize_$tool.log 2>&1; echo "rc=$?" >> gpurun_out/ev_sanitize_$tool.log
-done
 # launch list of the default bench command (device times per launch; shares, not absolutes)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_launches_default.csv python bench.py --steps 5 --warmup 3 --no-cpu --ncu off --legs none --tca 0 --graphconv 0 --no-e2e --no-cusparse > /dev/null 2>&1
 mkdir -p /tmp/ncu
