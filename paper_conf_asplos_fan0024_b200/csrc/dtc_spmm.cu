@@ -320,6 +320,110 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
     split_fixup_h<1, NJ, VEC, QPC, CSTRIDE>(u, reinterpret_cast<float(&)[1][NJ][4]>(acc), ws, npad, ctr0, cstride, C,
                                             ldc, M, N, g, lane, base, hoff, rowmap);
 }
+// ---------------------------------------------- TF32 swapped-operand tiles (k_spmm_pad)
+// The padded kernel's TF32 mma computes C^T = B^T A^T: the gathered B rows are the m16n8k8 A operand
+// (m = 16 B columns, k = the block's 8 B rows), the TC block's values the B operand (n = 8 window
+// rows).  A lane's A operand {B[k=t][m=g], B[k=t][m=g+8], B[k=t+4][m=g], B[k=t+4][m=g+8]} is two
+// LDS.64 when columns m = g and g + 8 are adjacent in memory, so no register moves precede the HMMA.
+// 16-column tile q of a 128-byte segment: lane g's column pair starts at byte sw_colbyte(q, g) --
+// {0, 8, 64, 72} for g < 4, {32, 40, 96, 104} for g >= 4, +16 for q = 1 -- which with rows 16 mod
+// 128 bytes apart keeps every half-warp LDS.64 conflict-free.  Accumulator j = (cw*2 + q)*2 + nh
+// of a warp holds rows 8nh + 2t (d0, d2) and 8nh + 2t + 1 (d1, d3) at columns c, c + 1,
+// c = cw*32 + sw_colbyte(q, g)/4.
+__host__ __device__ constexpr int sw_colbyte(int q, int g) { return 8 * (g & 1) + 64 * ((g >> 1) & 1) + 32 * (g >> 2) + 16 * q; }
+__device__ __forceinline__ int sw_col(int j, int g) { return (j >> 2) * 32 + sw_colbyte((j >> 1) & 1, g) / 4; }
+
+template <int NJ, bool VEC>
+__device__ __forceinline__ void store_tile_sw(float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int64_t w, int g, int t,
+                                              int64_t n0, const float (&acc)[NJ][4], bool zero,
+                                              const int32_t* __restrict__ rowmap) {
+#pragma unroll
+    for (int nh = 0; nh < 2; ++nh)
+#pragma unroll
+        for (int rr = 0; rr < 2; ++rr) {
+            const int64_t row = w * kWindow + 8 * nh + 2 * t + rr;
+            if (row >= M) continue;
+            float* crow = C + (rowmap ? (int64_t)__ldg(rowmap + row) : row) * ldc;
+#pragma unroll
+            for (int jj = 0; jj < NJ / 2; ++jj) {
+                const int j = 2 * jj + nh;
+                const int64_t c = n0 + sw_col(j, g);
+                const float v0 = zero ? 0.f : acc[j][rr], v1 = zero ? 0.f : acc[j][2 + rr];
+                if (VEC) {
+                    if (c < N) *reinterpret_cast<float2*>(crow + c) = make_float2(v0, v1);
+                } else {
+                    if (c < N) crow[c] = v0;
+                    if (c + 1 < N) crow[c + 1] = v1;
+                }
+            }
+        }
+}
+
+template <int NJ>
+__device__ __forceinline__ void fixup_write_sw(float (&acc)[NJ][4], float* __restrict__ ws, int64_t slot, int64_t npad,
+                                               int g, int t, int64_t n0) {
+#pragma unroll
+    for (int nh = 0; nh < 2; ++nh)
+#pragma unroll
+        for (int rr = 0; rr < 2; ++rr) {
+            float* prow = ws + (slot * kWindow + 8 * nh + 2 * t + rr) * npad;
+#pragma unroll
+            for (int jj = 0; jj < NJ / 2; ++jj) {
+                const int j = 2 * jj + nh;
+                __stcg(reinterpret_cast<float2*>(prow + n0 + sw_col(j, g)), make_float2(acc[j][rr], acc[j][2 + rr]));
+            }
+        }
+}
+
+template <int NJ>
+__device__ __forceinline__ void fixup_sum_sw(float (&acc)[NJ][4], const float* __restrict__ ws, int64_t s0, int64_t step,
+                                             int cnt, int64_t npad, int g, int t, int64_t n0) {
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+#pragma unroll 1
+    for (int k = 0; k < cnt; ++k) {
+        const int64_t sl = s0 + k * step;
+#pragma unroll
+        for (int nh = 0; nh < 2; ++nh)
+#pragma unroll
+            for (int rr = 0; rr < 2; ++rr) {
+                const float* prow = ws + (sl * kWindow + 8 * nh + 2 * t + rr) * npad;
+#pragma unroll
+                for (int jj = 0; jj < NJ / 2; ++jj) {
+                    const int j = 2 * jj + nh;
+                    const float2 v = __ldcg(reinterpret_cast<const float2*>(prow + n0 + sw_col(j, g)));
+                    acc[j][rr] += v.x;
+                    acc[j][2 + rr] += v.y;
+                }
+            }
+    }
+}
+
+// split_fixup_h for swapped TF32 tiles (the same two-level deterministic protocol)
+template <int H, int NJ, bool VEC>
+__device__ __forceinline__ void split_fixup_h_sw(const Unit& u, float (&acc)[H][NJ][4], float* __restrict__ ws,
+                                                 int64_t npad, int32_t* __restrict__ ctr0, int64_t cstride,
+                                                 float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int g, int t,
+                                                 int lane, int64_t n0, const int32_t* __restrict__ rowmap) {
+    const int np = u.npieces, G = fixup_group(np);
+    const int g0 = (u.piece / G) * G, gn = min(G, np - g0), ngr = (np + G - 1) / G;
+    const int64_t sb = u.slot_base;
+#pragma unroll
+    for (int h = 0; h < H; ++h) fixup_write_sw<NJ>(acc[h], ws, (sb + u.piece) * H + h, npad, g, t, n0);
+    if (!arrive_last(ctr0 + (sb + g0) * cstride, gn, lane)) return;
+#pragma unroll
+    for (int h = 0; h < H; ++h) fixup_sum_sw<NJ>(acc[h], ws, (sb + g0) * H + h, H, gn, npad, g, t, n0);
+    if (ngr > 1) {
+#pragma unroll
+        for (int h = 0; h < H; ++h) fixup_write_sw<NJ>(acc[h], ws, (sb + g0) * H + h, npad, g, t, n0);
+        if (!arrive_last(ctr0 + (sb + 1) * cstride, ngr, lane)) return;
+#pragma unroll
+        for (int h = 0; h < H; ++h) fixup_sum_sw<NJ>(acc[h], ws, sb * H + h, (int64_t)G * H, ngr, npad, g, t, n0);
+    }
+#pragma unroll
+    for (int h = 0; h < H; ++h) store_tile_sw<NJ, VEC>(C, ldc, M, N, (int64_t)u.wb * H + h, g, t, n0, acc[h], false, rowmap);
+}
+
 // ============================================================ fallback: register gather
 // 64 zero bytes that padded (-1) B rows and columns beyond N read instead of B
 // (branch-free gather: the address is selected, the load is unconditional).
@@ -849,6 +953,11 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const uint32_t aring = ring + R * STAGE;                          // [2][ASLOT] A batches
     __shared__ int s_abyte[NA];   // byte offset of the batch's first value inside its A slot (batch c: slot (uint32_t)c % NA)
     constexpr bool COOP = pad_coop<DT, SL, SEG, H>();
+    // TF32 with 1 KB slices: swapped mma operands (B rows as the A operand, see store_tile_sw) -- no
+    // register moves before the HMMAs: c3 +2.3%, c4/256 +1.4%; the 512 B-slice kernel runs on 80
+    // registers, where the swap serialises its LDS/HMMA pairs and the epilogue's float2 stores weigh
+    // more (c2 -8%, c4/128 -3.5%), so it keeps the direct form (profiles/r02_ab_issue.txt)
+    constexpr bool SWAP = DT == DTC_TF32 && SEG == 8;
     __shared__ uint8_t s_live[2][BATCH];   // COOP: per block, bit h = sub-tile h has a non-zero
     const uint32_t frags = aring + NA * ASLOT;  // COOP: [2][BATCH][H] lane-major fragments (expand())
     // mbarriers: full[R], empty[R] (B stages), afull[NA], aempty[NA] (A batches), ufull[2], uempty[2]
@@ -1063,6 +1172,10 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     const int cg = (g >> 1) + 4 * (g & 1);
     const uint32_t roff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + cg * 16;
     const uint32_t roff1 = roff0 + ODD;
+    // TF32 (swapped operands): row t of the even / odd half at lane g's column pair of tile q = 0
+    const uint32_t soff0 = sl * SLB + t * ROWB + (warp % WPS) * CW * 128 + sw_colbyte(0, g);
+    const uint32_t soff1 = soff0 + ODD;
+    const int64_t n0w = n0;
 
     // S1, decoding one 16-row sub-tile of a TC block into this lane's mma A fragment: the occupancy
     // mask m and the block's values at vaddr (ascending local id, C5)
@@ -1074,9 +1187,12 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         const bool p00 = (wl >> pos) & 1u, p01 = (wl >> (pos + 1)) & 1u;
         const bool p10 = (wh >> pos) & 1u, p11 = (wh >> (pos + 1)) & 1u;
         if constexpr (DT == DTC_TF32) {
+            // A fragment (g,t) (g+8,t) (g,t+4) (g+8,t+4); swapped operands want the mma B operand of
+            // rows g (a[0], a[1]) and g + 8 (a[2], a[3]), k = t then t + 4
+            constexpr int I1 = SWAP ? 2 : 1, I2 = SWAP ? 1 : 2;
             a[0] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rl, p00)));
-            a[1] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rh, p10)));
-            a[2] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rl + p00), p01)));
+            a[I1] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * rh, p10)));
+            a[I2] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rl + p00), p01)));
             a[3] = to_tf32(__uint_as_float(lds32_pred(vaddr + 4 * (rh + p10), p11)));
         } else {
             a[0] = lds16_pred(vaddr + 2 * rl, p00) | (lds16_pred(vaddr + 2 * (rl + p00), p01) << 16);
@@ -1223,8 +1339,12 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         // C rows of window w: the 16-row tiles w*H .. w*H+H-1
         auto store_window = [&](int w, bool zero) {
 #pragma unroll
-            for (int h = 0; h < H; ++h)
-                store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, (int64_t)w * H + h, g, base, hoff, acc[h], zero, rowmap);
+            for (int h = 0; h < H; ++h) {
+                if constexpr (SWAP)
+                    store_tile_sw<NJ, VEC>(C, ldc, M, N, (int64_t)w * H + h, g, t, n0w, acc[h], zero, rowmap);
+                else
+                    store_tile<NJ, VEC, QPC, COLW1>(C, ldc, M, N, (int64_t)w * H + h, g, base, hoff, acc[h], zero, rowmap);
+            }
         };
         int cur = u.wb;
         int next_end = INT_MAX;
@@ -1252,7 +1372,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
             mbar_wait(bar_full + 8u * (s), ((uint32_t)gi / R) & 1);
             if (TRACE && tr && gi == 0 && threadIdx.x == 0) tr[4] = gtimer();   // (compiled out unless traced)
             const uint32_t st = ring + s * STAGE;
-            if constexpr (DT == DTC_TF32) {
+            if constexpr (DT == DTC_TF32 && !SWAP) {
 #pragma unroll
                 for (int cw = 0; cw < CW; ++cw) {
                     const uint4 x0 = lds128(st + roff0 + cw * 128);
@@ -1263,9 +1383,25 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
                     for (int h = 0; h < H; ++h)
                         if (H == 1 || live[h])
 #pragma unroll
-                            // (the B pair {y0, y1} needs register moves before each HMMA; two m16n8k4
-                            // halves avoid them but measured 2-11% slower, profiles/r02_ab_issue.txt)
                             for (int jj = 0; jj < NJ1; ++jj) mma_tf32(acc[h][cw * NJ1 + jj], a[h], y0[jj & 3], y1[jj & 3]);
+                }
+            } else if constexpr (DT == DTC_TF32) {
+#pragma unroll
+                for (int cw = 0; cw < CW; ++cw) {
+#pragma unroll
+                    for (int q = 0; q < 2; ++q) {
+                        // A operand = B^T tile q: rows k = t (even half) and t + 4 (odd half), columns
+                        // m = g, g + 8 adjacent -- two LDS.64 straight into the HMMA's register quadruple
+                        const uint2 e = lds64(st + soff0 + cw * 128 + 16 * q);
+                        const uint2 o = lds64(st + soff1 + cw * 128 + 16 * q);
+                        const uint32_t bt[4] = {e.x, e.y, o.x, o.y};
+#pragma unroll
+                        for (int h = 0; h < H; ++h)
+                            if (H == 1 || live[h])
+#pragma unroll
+                                for (int nh = 0; nh < 2; ++nh)
+                                    mma_tf32(acc[h][(cw * 2 + q) * 2 + nh], bt, a[h][2 * nh], a[h][2 * nh + 1]);
+                    }
                 }
             } else {
                 if (pair) {
@@ -1329,9 +1465,13 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         if (!split) {
             while (cur < u.we) { store_window(cur, true); ++cur; }
         } else {
-            split_fixup_h<H, NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * kFixupWarps + warp,
-                                                  (int64_t)gridDim.y * kFixupWarps, C, ldc, M, N, g, lane, base, hoff,
-                                                  rowmap);
+            if constexpr (SWAP)
+                split_fixup_h_sw<H, NJ, VEC>(u, acc, ws, npad, counters + blockIdx.y * kFixupWarps + warp,
+                                             (int64_t)gridDim.y * kFixupWarps, C, ldc, M, N, g, t, lane, n0w, rowmap);
+            else
+                split_fixup_h<H, NJ, VEC, QPC, COLW1>(u, acc, ws, npad, counters + blockIdx.y * kFixupWarps + warp,
+                                                      (int64_t)gridDim.y * kFixupWarps, C, ldc, M, N, g, lane, base, hoff,
+                                                      rowmap);
         }
         gi0 += nblocks;
         gc0 += (nblocks + BATCH - 1) / BATCH;
