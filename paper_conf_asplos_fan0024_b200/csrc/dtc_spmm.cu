@@ -333,27 +333,47 @@ __device__ __forceinline__ void split_fixup(const Unit& u, float (&acc)[NJ][4], 
 __host__ __device__ constexpr int sw_colbyte(int q, int g) { return 8 * (g & 1) + 64 * ((g >> 1) & 1) + 32 * (g >> 2) + 16 * q; }
 __device__ __forceinline__ int sw_col(int j, int g) { return (j >> 2) * 32 + sw_colbyte((j >> 1) & 1, g) / 4; }
 
+// Vector path: lanes g and g^1 (lane ^ 4) hold columns [b, b+2) and [b+2, b+4) of tile q = 0 and
+// [b+4, b+8) of q = 1; one exchange gives the even lane q = 0's four columns and the odd lane q = 1's,
+// so every lane stores one float4 per (segment, row) -- whole 16-byte pieces, which matter when C is
+// pinned host memory written over PCIe (float2 stores halved the streaming e2e rate).
 template <int NJ, bool VEC>
 __device__ __forceinline__ void store_tile_sw(float* __restrict__ C, int64_t ldc, int64_t M, int64_t N, int64_t w, int g, int t,
                                               int64_t n0, const float (&acc)[NJ][4], bool zero,
                                               const int32_t* __restrict__ rowmap) {
+    const bool odd = g & 1;
 #pragma unroll
     for (int nh = 0; nh < 2; ++nh)
 #pragma unroll
         for (int rr = 0; rr < 2; ++rr) {
             const int64_t row = w * kWindow + 8 * nh + 2 * t + rr;
-            if (row >= M) continue;
-            float* crow = C + (rowmap ? (int64_t)__ldg(rowmap + row) : row) * ldc;
+            if (VEC) {
+                float4 v[NJ / 4];
 #pragma unroll
-            for (int jj = 0; jj < NJ / 2; ++jj) {
-                const int j = 2 * jj + nh;
-                const int64_t c = n0 + sw_col(j, g);
-                const float v0 = zero ? 0.f : acc[j][rr], v1 = zero ? 0.f : acc[j][2 + rr];
-                if (VEC) {
-                    if (c < N) *reinterpret_cast<float2*>(crow + c) = make_float2(v0, v1);
-                } else {
-                    if (c < N) crow[c] = v0;
-                    if (c + 1 < N) crow[c + 1] = v1;
+                for (int cw = 0; cw < NJ / 4; ++cw) {
+                    const int j0 = (cw * 2) * 2 + nh, j1 = (cw * 2 + 1) * 2 + nh;
+                    const float a0 = zero ? 0.f : acc[j0][rr], a1 = zero ? 0.f : acc[j0][2 + rr];
+                    const float b0 = zero ? 0.f : acc[j1][rr], b1 = zero ? 0.f : acc[j1][2 + rr];
+                    const float r0 = __shfl_xor_sync(0xffffffffu, odd ? a0 : b0, 4);
+                    const float r1 = __shfl_xor_sync(0xffffffffu, odd ? a1 : b1, 4);
+                    v[cw] = odd ? make_float4(r0, r1, b0, b1) : make_float4(a0, a1, r0, r1);
+                }
+                if (row >= M) continue;
+                float* crow = C + (rowmap ? (int64_t)__ldg(rowmap + row) : row) * ldc;
+#pragma unroll
+                for (int cw = 0; cw < NJ / 4; ++cw) {
+                    const int64_t c = n0 + cw * 32 + sw_colbyte(0, g & ~1) / 4 + (odd ? 4 : 0);
+                    if (c < N) *reinterpret_cast<float4*>(crow + c) = v[cw];
+                }
+            } else {
+                if (row >= M) continue;
+                float* crow = C + (rowmap ? (int64_t)__ldg(rowmap + row) : row) * ldc;
+#pragma unroll
+                for (int jj = 0; jj < NJ / 2; ++jj) {
+                    const int j = 2 * jj + nh;
+                    const int64_t c = n0 + sw_col(j, g);
+                    if (c < N) crow[c] = zero ? 0.f : acc[j][rr];
+                    if (c + 1 < N) crow[c + 1] = zero ? 0.f : acc[j][2 + rr];
                 }
             }
         }

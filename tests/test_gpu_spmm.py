@@ -95,12 +95,13 @@ def test_p6_column_independence(dtype):
 
 @pytest.mark.parametrize("dtype", ["tf32", "fp16"])
 @pytest.mark.parametrize("U", [1, 2, 5])
-def test_split_windows_fixup(U, dtype):
-    """Tiny work units force many split windows: the deterministic fixup path."""
+@pytest.mark.parametrize("N", [96, 256, 258])
+def test_split_windows_fixup(U, dtype, N):
+    """Tiny work units force many split windows: the deterministic fixup path (N = 256 / 258: the
+    TF32 1 KB-slice kernel's transposed tiles, vector and scalar C stores)."""
     cfg = configs.get("c1")
     rp, ci = configs.make_pattern(cfg)
     v = configs.make_values(cfg, len(ci))
-    N = 96
     B = datagen.uniform(4, 2, cfg.K * N).reshape(cfg.K, N)
     if dtype == "fp16":
         v, B = v.astype(np.float16), B.astype(np.float16)
@@ -127,6 +128,27 @@ def test_deterministic_and_overwrites_everything():
     torch.cuda.synchronize()
     assert not torch.isnan(C1).any()
     assert torch.equal(C1, C2)
+
+
+@pytest.mark.parametrize("dtype", ["tf32", "fp16"])
+@pytest.mark.parametrize("N", [258, 300])
+def test_misaligned_c_wide_rows(dtype, N):
+    """Aligned B (the TMA path with 1 KB slices for TF32), C with an odd leading dimension and start:
+    the scalar stores of the transposed TF32 tiles, ragged last column group."""
+    torch = _torch()
+    M, K = 300, 400
+    rp, ci = datagen.random_csr(M, K, 0.05, 11)
+    v = datagen.uniform(11, 1, len(ci))
+    B = datagen.uniform(11, 2, K * N).reshape(K, N)
+    if dtype == "fp16":
+        v, B = v.astype(np.float16), B.astype(np.float16)
+    f = build(M, K, rp, ci, v, dtype=dtype)
+    Cbig = torch.full((M, N + 5), float("nan"), device="cuda")
+    C = Cbig[:, 1:1 + N]                 # ldc = N + 5, misaligned
+    f.spmm(dev(B), C)
+    torch.cuda.synchronize()
+    check_tol(C.cpu().numpy(), M, K, rp, ci, v, B, dtype)
+    assert torch.isnan(Cbig[:, :1]).all() and torch.isnan(Cbig[:, 1 + N:]).all()
 
 
 @pytest.mark.parametrize("dtype", ["tf32", "fp16"])
