@@ -794,8 +794,10 @@ template <int SEG> constexpr int pad_row_bytes() { return SEG * 128 + 16; }
 template <int SEG> constexpr int pad_odd_off() { return (4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_slice_bytes() { return (pad_odd_off<SEG>() + 4 * pad_row_bytes<SEG>() + 127) / 128 * 128; }
 template <int SEG> constexpr int pad_tx_bytes() { return 8 * pad_row_bytes<SEG>(); }
-static_assert(pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16, "row pitch must be 16 mod 128");
-static_assert(pad_row_bytes<4>() % 8 == 0 && pad_row_bytes<8>() % 8 == 0, "row pitch: whole 8-byte elements");
+static_assert(pad_row_bytes<2>() % 128 == 16 && pad_row_bytes<4>() % 128 == 16 && pad_row_bytes<8>() % 128 == 16,
+              "row pitch must be 16 mod 128");
+static_assert(pad_row_bytes<2>() % 8 == 0 && pad_row_bytes<4>() % 8 == 0 && pad_row_bytes<8>() % 8 == 0,
+              "row pitch: whole 8-byte elements");
 // B ring depth (stages of SL slices); measured flat between 3 and 6 once the A side is staged
 // (profiles/r01_design_evidence.md), and 6-10 stages with 8-block A batches 4-22% slower than 4
 // (profiles/r02_ab_issue.txt): deeper rings only cost CTAs per SM.  -DDTC_PAD_STAGES=k overrides
@@ -1529,7 +1531,7 @@ static bool make_bmap_pad(CUtensorMap* map, const void* B, int64_t K, int64_t N,
     if (!enc) return false;
     const int elt = elt_size(dtype);
     if (seg == 8 && te != 8) return false;
-    const int row_bytes = seg == 4 ? pad_row_bytes<4>() : pad_row_bytes<8>();
+    const int row_bytes = seg == 2 ? pad_row_bytes<2>() : seg == 4 ? pad_row_bytes<4>() : pad_row_bytes<8>();
     cuuint64_t dims[2] = {(cuuint64_t)(N * elt / te), (cuuint64_t)K};
     cuuint64_t strides[1] = {(cuuint64_t)(ldb * elt)};
     cuuint32_t box[2] = {(cuuint32_t)(row_bytes / te), 1};
@@ -1549,7 +1551,7 @@ struct LaunchArgs {
     int gy;
     int64_t npad;
     cudaStream_t s;
-    int seg;   // padded path: 128-byte segments per slice (4 or 8)
+    int seg;   // padded path: 128-byte segments per slice (2, 4 or 8)
     int te;    // padded path: TMA element bytes (4 or 8)
 };
 
@@ -1714,21 +1716,26 @@ static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
 template <int DT, bool VEC, int H>
 static cudaError_t dispatch_pad_h(int slices, const LaunchArgs& a, const CUtensorMap& map) {
     if (a.seg == 8) return slices >= 2 ? launch_pad<DT, 2, 8, VEC, H>(a, map) : launch_pad<DT, 1, 8, VEC, H>(a, map);
+    if (a.seg == 2) return launch_pad<DT, 1, 2, VEC, H>(a, map);
     return slices >= 2 ? launch_pad<DT, 2, 4, VEC, H>(a, map) : launch_pad<DT, 1, 4, VEC, H>(a, map);
 }
 template <int DT, bool VEC>
 static cudaError_t dispatch_pad(int slices, const LaunchArgs& a, const CUtensorMap& map) {
     if (DT == DTC_TF32 && a.h->window_h == 32)
-        return a.seg == 8 ? launch_pad<DTC_TF32, 1, 8, VEC, 2>(a, map) : launch_pad<DTC_TF32, 1, 4, VEC, 2>(a, map);
+        return a.seg == 8 ? launch_pad<DTC_TF32, 1, 8, VEC, 2>(a, map)
+             : a.seg == 2 ? launch_pad<DTC_TF32, 1, 2, VEC, 2>(a, map)
+                          : launch_pad<DTC_TF32, 1, 4, VEC, 2>(a, map);
     return dispatch_pad_h<DT, VEC, 1>(slices, a, map);
 }
 
 // Padded-path geometry for N columns: 1 KB slices (8-byte TMA elements) when a B row holds >= 1 KB,
-// else 512 B; <= 2 slices (seg/2 consumer warps each) per CTA.
+// 256 B slices (one consumer warp) when it holds <= 256 B -- a 512 B slice would leave half its
+// consumer warps computing columns past N -- else 512 B; <= 2 slices (seg/2 consumer warps each)
+// per CTA.
 PadGeometry pad_geometry(int dtype, int64_t N, int slice_bytes) {
     const int elt = elt_size(dtype);
     PadGeometry g;
-    g.seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : 4;
+    g.seg = ((N * elt) >= 1024 && (N * elt) % 8 == 0) ? 8 : (N * elt) <= 256 ? 2 : 4;
     if (slice_bytes == 512) g.seg = 4;
     if (slice_bytes == 1024 && (N * elt) % 8 == 0) g.seg = 8;
     const int64_t slice_cols = g.seg * 128 / elt;
@@ -1753,7 +1760,7 @@ int pad_occupancy(int dtype, int64_t N, int window_h) {
         if (smem > 48 * 1024 &&
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
             return -1;
-        const int thr = (sl * seg / (seg == 8 ? pad_cw<8>() : pad_cw<4>()) + 1) * 32;
+        const int thr = (sl * seg / (seg == 8 ? pad_cw<8>() : pad_cw<4>()) + 1) * 32;   // (pad_cw<2>() == pad_cw<4>())
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, kern, thr, smem) != cudaSuccess) return -1;
         return v;
     };
@@ -1762,12 +1769,14 @@ int pad_occupancy(int dtype, int64_t N, int window_h) {
         if (g.seg == 8)                                                                                             \
             return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 8, true, H>, 2, 8, pad_smem_bytes<2, 8, H, DT>())               \
                                  : occ(k_spmm_pad<DT, 1, 8, true, H>, 1, 8, pad_smem_bytes<1, 8, H, DT>());              \
+        if (g.seg == 2) return occ(k_spmm_pad<DT, 1, 2, true, H>, 1, 2, pad_smem_bytes<1, 2, H, DT>());               \
         return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 4, true, H>, 2, 4, pad_smem_bytes<2, 4, H, DT>())                   \
                              : occ(k_spmm_pad<DT, 1, 4, true, H>, 1, 4, pad_smem_bytes<1, 4, H, DT>());                  \
     } while (0)
     if (dtype == DTC_FP16) DTC_OCC(DTC_FP16, 1);
     if (window_h == 32) {   // one slice per CTA (see spmm_launch)
         if (g.seg == 8) return occ(k_spmm_pad<DTC_TF32, 1, 8, true, 2>, 1, 8, pad_smem_bytes<1, 8, 2>());
+        if (g.seg == 2) return occ(k_spmm_pad<DTC_TF32, 1, 2, true, 2>, 1, 2, pad_smem_bytes<1, 2, 2>());
         return occ(k_spmm_pad<DTC_TF32, 1, 4, true, 2>, 1, 4, pad_smem_bytes<1, 4, 2>());
     }
     DTC_OCC(DTC_TF32, 1);
