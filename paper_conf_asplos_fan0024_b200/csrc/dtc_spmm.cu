@@ -869,14 +869,19 @@ template <int DT, int SL, int SEG, int H> constexpr int pad_aslot() {
 #ifndef DTC_PAD_SEG8_CW
 #define DTC_PAD_SEG8_CW 2
 #endif
-template <int SEG> constexpr int pad_cw() { return SEG == 8 ? DTC_PAD_SEG8_CW : 2; }
-template <int SL, int SEG> constexpr int pad_consumers() { return SL * SEG / pad_cw<SEG>(); }
+#ifndef DTC_PAD_FP16_CW
+#define DTC_PAD_FP16_CW 2
+#endif
+template <int DT, int SEG> constexpr int pad_cw() {
+    return SEG == 8 ? DTC_PAD_SEG8_CW : (DT == DTC_FP16 && SEG == 4 ? DTC_PAD_FP16_CW : 2);
+}
+template <int DT, int SL, int SEG> constexpr int pad_consumers() { return SL * SEG / pad_cw<DT, SEG>(); }
 #ifndef DTC_PAD_COOP_FORCE
 #define DTC_PAD_COOP_FORCE -1
 #endif
 template <int DT, int SL, int SEG, int H>
 constexpr bool pad_coop() {
-    return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || pad_consumers<SL, SEG>() >= 4 || H > 1);
+    return DTC_PAD_COOP_FORCE >= 0 ? DTC_PAD_COOP_FORCE == 1 : (DT == DTC_FP16 || pad_consumers<DT, SL, SEG>() >= 4 || H > 1);
 }
 template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
     return pad_coop<DT, SL, SEG, H>() ? 2 * pad_batch<DT, SL, SEG, H>() * H * 32 * Traits<DT>::FRAG_WORDS * 4 : 0;
@@ -893,6 +898,9 @@ constexpr size_t pad_smem_bytes() {
 #ifndef DTC_PAD_CW1_REGS
 #define DTC_PAD_CW1_REGS 72
 #endif
+#ifndef DTC_PAD_FP16_REGS
+#define DTC_PAD_FP16_REGS 128
+#endif
 template <int DT, int SL, int SEG, int H>
 constexpr int pad_maxregs() {
     if (H > 1) return SL >= 2 ? 112 : 128;   // two 16-row accumulator tiles per thread
@@ -900,7 +908,7 @@ constexpr int pad_maxregs() {
 #ifdef DTC_PAD_MAXREGS
     return DTC_PAD_MAXREGS;
 #else
-    return DT == DTC_FP16 ? 128 : (pad_slim<DT, SL, SEG, H>() ? 96 : 104);
+    return DT == DTC_FP16 ? DTC_PAD_FP16_REGS : (pad_slim<DT, SL, SEG, H>() ? 96 : 104);
 #endif
 }
 
@@ -940,8 +948,8 @@ __device__ __forceinline__ uint32_t lds16_pred(uint32_t a, bool p) {
 template <int DT, int SL, int SEG, bool VEC, int H, bool TRACE = false>
 // (min-blocks form of the register cap: measured 8-13% faster than __maxnreg__ with the same cap,
 // profiles/r02_ab_launch_bounds.txt)
-__global__ void __launch_bounds__((pad_consumers<SL, SEG>() + 1) * 32,
-                                  65536 / ((pad_consumers<SL, SEG>() + 1) * 32 * pad_maxregs<DT, SL, SEG, H>()))
+__global__ void __launch_bounds__((pad_consumers<DT, SL, SEG>() + 1) * 32,
+                                  65536 / ((pad_consumers<DT, SL, SEG>() + 1) * 32 * pad_maxregs<DT, SL, SEG, H>()))
 k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ units, const int32_t* __restrict__ rwo,
            const int32_t* __restrict__ tco, const uint4* __restrict__ mask, const int32_t* __restrict__ atob,
            const void* __restrict__ avals, float* __restrict__ C, int64_t ldc, int64_t M, int64_t N,
@@ -959,7 +967,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
         tr[1] = smid();
         tr[2] = gtimer();
     }
-    constexpr int CW = pad_cw<SEG>();          // 128-byte segments per consumer warp
+    constexpr int CW = pad_cw<DT, SEG>();      // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
     constexpr int R = pad_stages<SL>();
     constexpr int G = pad_issue<DT, SL, SEG, H>();
@@ -1662,7 +1670,7 @@ static cudaError_t lpt_units(dtc_format* h, cudaStream_t s) {
 template <int DT, int SL, int SEG, bool VEC, int H>
 static cudaError_t launch_pad(const LaunchArgs& a, const CUtensorMap& map) {
     constexpr size_t smem = pad_smem_bytes<SL, SEG, H, DT>();
-    constexpr int threads = (pad_consumers<SL, SEG>() + 1) * 32;
+    constexpr int threads = (pad_consumers<DT, SL, SEG>() + 1) * 32;
     static KernelState ks;
     const int per_sm = kernel_setup(k_spmm_pad<DT, SL, SEG, VEC, H>, threads, smem, ks, a.h->device);
     if (per_sm < 0) {
@@ -1754,30 +1762,29 @@ int pad_occupancy(int dtype, int64_t N, int window_h) {
     const PadGeometry g = pad_geometry(dtype, N, 0);
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return -1; }
-    auto occ = [&](auto kern, int sl, int seg, size_t smem) -> int {
+    auto occ = [&](auto kern, int thr, size_t smem) -> int {
         // (every k_spmm_pad instantiation has the same type, so no per-type static cache here)
         int v = 0;
         if (smem > 48 * 1024 &&
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
             return -1;
-        const int thr = (sl * seg / (seg == 8 ? pad_cw<8>() : pad_cw<4>()) + 1) * 32;   // (pad_cw<2>() == pad_cw<4>())
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, kern, thr, smem) != cudaSuccess) return -1;
         return v;
     };
 #define DTC_OCC(DT, H)                                                                                              \
     do {                                                                                                            \
         if (g.seg == 8)                                                                                             \
-            return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 8, true, H>, 2, 8, pad_smem_bytes<2, 8, H, DT>())               \
-                                 : occ(k_spmm_pad<DT, 1, 8, true, H>, 1, 8, pad_smem_bytes<1, 8, H, DT>());              \
-        if (g.seg == 2) return occ(k_spmm_pad<DT, 1, 2, true, H>, 1, 2, pad_smem_bytes<1, 2, H, DT>());               \
-        return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 4, true, H>, 2, 4, pad_smem_bytes<2, 4, H, DT>())                   \
-                             : occ(k_spmm_pad<DT, 1, 4, true, H>, 1, 4, pad_smem_bytes<1, 4, H, DT>());                  \
+            return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 8, true, H>, (pad_consumers<DT, 2, 8>() + 1) * 32, pad_smem_bytes<2, 8, H, DT>())               \
+                                 : occ(k_spmm_pad<DT, 1, 8, true, H>, (pad_consumers<DT, 1, 8>() + 1) * 32, pad_smem_bytes<1, 8, H, DT>());              \
+        if (g.seg == 2) return occ(k_spmm_pad<DT, 1, 2, true, H>, (pad_consumers<DT, 1, 2>() + 1) * 32, pad_smem_bytes<1, 2, H, DT>());               \
+        return g.slices >= 2 ? occ(k_spmm_pad<DT, 2, 4, true, H>, (pad_consumers<DT, 2, 4>() + 1) * 32, pad_smem_bytes<2, 4, H, DT>())                   \
+                             : occ(k_spmm_pad<DT, 1, 4, true, H>, (pad_consumers<DT, 1, 4>() + 1) * 32, pad_smem_bytes<1, 4, H, DT>());                  \
     } while (0)
     if (dtype == DTC_FP16) DTC_OCC(DTC_FP16, 1);
     if (window_h == 32) {   // one slice per CTA (see spmm_launch)
-        if (g.seg == 8) return occ(k_spmm_pad<DTC_TF32, 1, 8, true, 2>, 1, 8, pad_smem_bytes<1, 8, 2>());
-        if (g.seg == 2) return occ(k_spmm_pad<DTC_TF32, 1, 2, true, 2>, 1, 2, pad_smem_bytes<1, 2, 2>());
-        return occ(k_spmm_pad<DTC_TF32, 1, 4, true, 2>, 1, 4, pad_smem_bytes<1, 4, 2>());
+        if (g.seg == 8) return occ(k_spmm_pad<DTC_TF32, 1, 8, true, 2>, (pad_consumers<DTC_TF32, 1, 8>() + 1) * 32, pad_smem_bytes<1, 8, 2>());
+        if (g.seg == 2) return occ(k_spmm_pad<DTC_TF32, 1, 2, true, 2>, (pad_consumers<DTC_TF32, 1, 2>() + 1) * 32, pad_smem_bytes<1, 2, 2>());
+        return occ(k_spmm_pad<DTC_TF32, 1, 4, true, 2>, (pad_consumers<DTC_TF32, 1, 4>() + 1) * 32, pad_smem_bytes<1, 4, 2>());
     }
     DTC_OCC(DTC_TF32, 1);
 #undef DTC_OCC
