@@ -197,7 +197,8 @@ int dtc_spmm_launches_per_call(void);
  *   DTC_OPT_HOST_CHUNKS    dtc_spmm_host column chunks, 0 = auto, 1..16.
  *   DTC_OPT_HOST_ZERO_COPY dtc_spmm_host stores C straight into pinned mapped C_host:
  *                          -1 = auto (when the format is larger than B), 0 = off, 1 = on.
- *   DTC_OPT_SLICE_BYTES    padded kernel row slice per gather4 op: 0 auto, 512 or 1024.
+ *   DTC_OPT_SLICE_BYTES    padded kernel row slice per gather4 op: 0 auto (1024 when a B row holds
+ *                          >= 1 KB, 256 when it holds <= 256 B, else 512), 512 or 1024.
  *   DTC_OPT_LAST_KERNEL    read-only: kernel the last dtc_spmm ran (1 register gather, 4 padded).
  *   DTC_OPT_LAST_HOST_MODE read-only: last dtc_spmm_host: 2 * column chunks + (1 if C was stored
  *                          zero-copy into host memory, i.e. no device-to-host copy).
