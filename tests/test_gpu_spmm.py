@@ -232,6 +232,24 @@ def test_tall_windows_full_size(name, N, parity_report):
     parity_report[f"{name} N={N} {cfg.dtype} tall32"] = (worst, cfg.M * N)
 
 
+@pytest.mark.parametrize("N", [8, 33, 64, 100])
+@pytest.mark.parametrize("U", [0, 2])
+def test_tall_windows_narrow_rows(N, U):
+    """32-row windows on the 256 B and 512 B slice kernels (B rows <= 256 B, ragged), with and
+    without forced splits: C within tolerance of O1, and integer inputs bit-exact."""
+    cfg = configs.get("c1")
+    rp, ci = configs.make_pattern(cfg)
+    v = configs.make_values(cfg, len(ci))
+    B = datagen.uniform(9, 2, cfg.K * N).reshape(cfg.K, N)
+    f = build(cfg.M, cfg.K, rp, ci, v, dtype="tf32", window_rows=32, unit_blocks=U)
+    check_tol(spmm(f, B), cfg.M, cfg.K, rp, ci, v, B, "tf32")
+    vi = np.rint(v * 4).astype(np.float32)
+    Bi = np.rint(B * 4).astype(np.float32)
+    fi = build(cfg.M, cfg.K, rp, ci, vi, dtype="tf32", window_rows=32, unit_blocks=U)
+    Cr, _ = oracle.spmm(cfg.M, cfg.K, rp, ci, vi, Bi)
+    assert np.array_equal(spmm(fi, Bi).astype(np.float64), Cr)
+
+
 @pytest.mark.parametrize("name,N", [("c3", 256), ("c3h", 256), ("c4", 128), ("c5", 512)])
 def test_p2_integer_full_size_exact(name, N, parity_report):
     """P2 at full size: integer A and B (|a|,|b| <= 2 -> every product and partial sum is exact in
