@@ -852,6 +852,16 @@ template <int DT, int SL, int SEG, int H> constexpr int pad_batch() {
     return pad_slim<DT, SL, SEG, H>() ? kPadBatch / 2 : kPadBatch / H;
 }
 static_assert(kPadBatch % 8 == 0, "first records hold the A range of the first 8 and 16 blocks");
+// B ring depth per geometry: 6 stages for FP16 512 B-slice CTAs (c3h +2.7%; they stay at 5 CTAs/SM,
+// limited by registers, with 44 KB of shared memory), pad_stages<SL> elsewhere (deeper rings cost
+// the TF32 kernels CTAs per SM, and the FP16 256 B-slice kernel 11%; profiles/r02_ab_issue.txt)
+template <int DT, int SL, int SEG, int H> constexpr int pad_stages_g() {
+#ifdef DTC_PAD_STAGES
+    return DTC_PAD_STAGES;
+#else
+    return (DT == DTC_FP16 && SL == 1 && SEG == 4) ? 6 : pad_stages<SL>();
+#endif
+}
 // (values of one block: at most 16H x 8 elements of the handle's dtype)
 template <int DT, int SL, int SEG, int H> constexpr int pad_aval_bytes() {
     return pad_batch<DT, SL, SEG, H>() * 128 * H * (DT == DTC_FP16 ? 2 : 4) + 128;
@@ -891,7 +901,7 @@ template <int DT, int SL, int SEG, int H> constexpr int pad_frag_bytes() {
 template <int DT, int SL, int SEG, int H> constexpr int pad_aslots() { return 2; }
 template <int SL, int SEG, int H = 1, int DT = DTC_TF32>
 constexpr size_t pad_smem_bytes() {
-    return (size_t)pad_stages<SL>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<DT, SL, SEG, H>() +
+    return (size_t)pad_stages_g<DT, SL, SEG, H>() * SL * pad_slice_bytes<SEG>() + pad_aslots<DT, SL, SEG, H>() * pad_aslot<DT, SL, SEG, H>() +
            pad_frag_bytes<DT, SL, SEG, H>() + 128 + 256;   // + alignment slack + mbarriers
 }
 // register cap (sets CTAs per SM); -DDTC_PAD_MAXREGS=r overrides for sweeps
@@ -969,7 +979,7 @@ k_spmm_pad(const __grid_constant__ CUtensorMap bmap, const Unit* __restrict__ un
     }
     constexpr int CW = pad_cw<DT, SEG>();      // 128-byte segments per consumer warp
     constexpr int NJ = NJ1 * CW, QPC = NJ1 / 4;   // QPC quads per segment, segments COLW1 apart
-    constexpr int R = pad_stages<SL>();
+    constexpr int R = pad_stages_g<DT, SL, SEG, H>();
     constexpr int G = pad_issue<DT, SL, SEG, H>();
     constexpr int WPS = SEG / CW;              // consumer warps per slice
     constexpr int ROWB = pad_row_bytes<SEG>(), ODD = pad_odd_off<SEG>(), SLB = pad_slice_bytes<SEG>();
