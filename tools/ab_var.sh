@@ -14,7 +14,7 @@ for r in rows: print('$lab', *r)
 }
 for rep in 1 2; do
   for v in default ${VARS}; do
-    if [ $v = default ]; then L=""; else L="DTC_LIBRARY=$PWD/${VDIR:-build_variants}/$v/libdtc.so"; fi
+    if [ $v = default ]; then L=""; else L="DTC_LIBRARY=$PWD/${VDIR:-vbuild}/$v/libdtc.so"; fi
     run $v $L $B --legs ${LEGS:-c2,c4:128,c4:256,c5} 2>/dev/null
   done
 done
